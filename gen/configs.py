@@ -1,0 +1,68 @@
+"""The five BASELINE.json workloads as plain data.
+
+No method arithmetic lives here: only bounds, horizons, controller constants and
+the workload recipe (cap schedule, demand kind, seeds).  Both the oracle wrapper
+(oracle/oracle.py) and the product binding read these dictionaries.
+
+Citations: P:NNN = /root/reference/PAPER.md line.
+"""
+from __future__ import annotations
+
+import copy
+
+# Knob classes (Q15): CPU 1.1-2.4 GHz in 100 MHz steps, V100-class
+# GPU 435-1350 MHz (nvidia-smi -ac 877,435-1350) on 11 levels (91.5 MHz).
+CPU_KNOB = dict(f_min=1100.0, f_max=2400.0, n_levels=14, sweep_base=3)  # base 1400 MHz
+GPU_KNOB = dict(f_min=435.0, f_max=1350.0, n_levels=11, sweep_base=0)   # base = lowest level
+
+# Controller constants (Q1, Q4, Q6, Q8, Q21; P = 8 / M = 2 from P:264; gamma P:190)
+CONTROLLER = dict(q=1.0, r0=1e-4, theta_min=0.05, lam=0.95, rho=100.0, a_lo=0.25, a_hi=4.0,
+                  a_floor=1e-3, gamma=0.91, noise_std=11.0, substeps=4)
+
+_BASE_WORKLOAD = dict(n_caps=1, demand_kind=1, demand_frac=0.7, cap_frac0=0.5, cap_frac_rand=0.0,
+                      cap_frac_step=0.0, cap_period=0, cap_lo=0, cap_hi=0, cap_mult=1.0,
+                      hierarchical=False)
+
+CONFIGS = {
+    # 1 server, 1 CPU + 2 GPUs, P/M = 4/2, 200 periods, fixed cap
+    1: dict(n_servers=1, n_gpus=2, P=4, M=2, periods=200, seed=1,
+            workload=dict(demand_kind=0, demand_frac=0.7, cap_frac0=0.6)),
+    # 1,024 servers, 1 CPU + 4 GPUs, 8/2, 1000 periods, step changes in cap
+    # (800 -> 900 -> 800 W analogue of Fig. 10: x 900/800 in [40, 80) mod 200)
+    2: dict(n_servers=1024, n_gpus=4, P=8, M=2, periods=1000, seed=2,
+            workload=dict(cap_frac0=0.45, cap_period=200, cap_lo=40, cap_hi=80, cap_mult=1.125)),
+    # 65,536 servers, 1 CPU + 8 GPUs (9 knobs), 8/3, 1000 periods, throughput-driven weights
+    3: dict(n_servers=65536, n_gpus=8, P=8, M=3, periods=1000, seed=3,
+            workload=dict(cap_frac0=0.3, cap_frac_rand=0.5)),
+    # 1,048,576 servers sharded over 8 GPUs, hierarchical rack budget (Q16)
+    4: dict(n_servers=1048576, n_gpus=8, P=8, M=2, periods=1000, seed=4,
+            workload=dict(hierarchical=True, rack=16, block=1024, cluster_frac=0.55,
+                          rack_frac=0.9)),
+    # cap sweep: 262,144 servers x 32 caps x 2,000 periods (Fig. 6 analogue)
+    5: dict(n_servers=262144, n_gpus=3, P=8, M=2, periods=2000, seed=5,
+            workload=dict(n_caps=32, cap_frac0=0.0, cap_frac_step=1.0 / 32.0)),
+}
+
+
+def knobs(n_gpus: int) -> list[dict]:
+    """Knob list: knob 0 = CPU, knobs 1..n_gpus = GPUs (paper order)."""
+    return [dict(CPU_KNOB)] + [dict(GPU_KNOB) for _ in range(n_gpus)]
+
+
+def get(cfg: int, **overrides) -> dict:
+    """Full description of config `cfg` (1..5) with optional overrides."""
+    c = copy.deepcopy(CONFIGS[cfg])
+    wl = dict(_BASE_WORKLOAD)
+    wl.update(c.pop("workload"))
+    c["workload"] = wl
+    c["controller"] = dict(CONTROLLER)
+    c["cfg"] = cfg
+    for k, v in overrides.items():
+        if k in c["controller"]:
+            c["controller"][k] = v
+        elif k in wl:
+            wl[k] = v
+        else:
+            c[k] = v
+    c["knobs"] = knobs(c["n_gpus"])
+    return c

@@ -1,0 +1,140 @@
+/*
+ * capgpu_oracle.h -- plain, slow, single-threaded CPU oracle of the CapGPU hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load or call this library.  The
+ * product path (paper_conf_icpp_masw25_b200/) never links, imports or executes it.
+ * It shares no code with the CUDA path except the seeded input generator
+ * gen/capgpu_gen.h (no method arithmetic lives there).
+ *
+ * Every function follows PAPER.md (cited "P:NNN" = /root/reference/PAPER.md line)
+ * or, where the paper is silent, the reading listed in DESIGN.md §2 (Q1..Q20).
+ * Floating point is IEEE fp64 compiled with -O2 -fno-fast-math -ffp-contract=off.
+ *
+ * Pins (tests/test_oracle_*.py): see DESIGN.md §4 for which pin covers which
+ * function.  Functions without an independent pin say "parity unpinned".
+ */
+#ifndef CAPGPU_ORACLE_H
+#define CAPGPU_ORACLE_H
+
+#include <stdint.h>
+
+#define ORA_MAXN 16
+#define ORA_MAXM 8
+#define ORA_MAXL 32
+#define ORA_MAXS 8
+
+/* per-server status bits (same meaning as include/capgpu.h) */
+#define ORA_ST_CAP_INFEASIBLE 1u
+#define ORA_ST_SLO_INFEASIBLE 2u
+#define ORA_ST_SOLVER_CAP 4u
+#define ORA_ST_NONFINITE 8u
+
+typedef struct {
+  int32_t n;         /* knobs N = 1 + n_gpus; knob 0 = CPU */
+  int32_t P, M;      /* prediction / control horizon */
+  int32_t substeps;  /* S: delta-sigma sub-steps per control period */
+  int32_t n_levels[ORA_MAXN];
+  int32_t sweep_base[ORA_MAXN]; /* base level index held during the sweep */
+  double f_min[ORA_MAXN], f_max[ORA_MAXN], f_lo[ORA_MAXN], r0[ORA_MAXN];
+  double q;          /* Q(i) = q (Q6) */
+  double theta_min;  /* Q8 */
+  double lambda;     /* forgetting factor of the online LS (Q1) */
+  double rho;        /* ridge toward A0 (Q1) */
+  double a_lo, a_hi; /* clamp of Ahat to [a_lo, a_hi] * A0 (Q4) */
+  double a_floor;    /* positivity guard on identified A0 (Q21) */
+  double gamma;      /* latency exponent */
+  double noise_std;  /* meter noise sigma (W) */
+  uint64_t seed;
+} ora_cfg;
+
+typedef struct {
+  int32_t periods;      /* control periods to run */
+  int32_t n_caps;       /* instances per server (cfg 5: 32) */
+  int32_t demand_kind;  /* 0 = constant frac, 1 = bursty */
+  double demand_frac;   /* constant demand fraction (cfg 1: 0.7) */
+  double cap_frac0, cap_frac_rand, cap_frac_step;
+  int64_t cap_period, cap_lo, cap_hi; /* step schedule */
+  double cap_mult;
+} ora_workload;
+
+/* per-instance summary over the last 80 % of periods */
+typedef struct {
+  double sum_p, sumsq_p, max_p, sum_theta;
+  int32_t n_window, n_viol;
+  int32_t act_count[ORA_MAXM]; /* periods where block t had >= 1 active bound */
+} ora_summary;
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- frequency grid (Q15): level(l) = f_min + l*step, mid(l) = f_min + (l+0.5)*step */
+void ora_levels(const ora_cfg *c, int j, double *level, double *mid, double *g);
+
+/* ---- S0 identification */
+int ora_identify_ls(int n, int rows, const double *F, const double *p, double *A, double *C, double *r2);
+int ora_sweep_rows(const ora_cfg *c, uint64_t server, int noisy, double *F, double *p);
+int ora_sweep_nrows(const ora_cfg *c);
+int ora_identify_server(const ora_cfg *c, uint64_t server, double *A0, double *C0, double *r2);
+
+/* ---- S1 model update (Eq. 5, LS P:173; online form Q1-Q4) */
+typedef struct {
+  double w, mu_f[ORA_MAXN], mu_p;
+  double S_ff[ORA_MAXN][ORA_MAXN], S_fp[ORA_MAXN];
+} ora_model;
+void ora_model_reset(ora_model *m);
+void ora_model_push(const ora_cfg *c, ora_model *m, const double *f, double p);
+void ora_model_solve(const ora_cfg *c, const ora_model *m, const double *A0, double *Ahat);
+void ora_model_definition(const ora_cfg *c, int count, const double *F_hist, const double *p_hist,
+                          const double *A0, double *Ahat);
+
+/* ---- S2 weights (Q8-Q10) */
+void ora_weights(const ora_cfg *c, const double *thr, const double *thr_max, double *theta,
+                 double *R, int8_t *rank);
+
+/* ---- S3 MPC (Eq. 9-10a; Q11-Q13, Q17, Q19) */
+int ora_block_weights(const ora_cfg *c, double *ct);
+int ora_mpc_stacked(const ora_cfg *c, const double *Ahat, const double *R, double beta,
+                    const double *lo, const double *hi, const double *m, double *u,
+                    uint32_t *active, uint32_t *tie, int *iters);
+int ora_mpc_bruteforce(const ora_cfg *c, const double *Ahat, const double *R, double beta,
+                       const double *lo, const double *hi, const double *m, double *u);
+double ora_mpc_cost(const ora_cfg *c, const double *Ahat, const double *R, double beta,
+                    const double *m, const double *u);
+void ora_mpc_classify(const ora_cfg *c, const double *Ahat, const double *R, double beta,
+                      const double *lo, const double *hi, const double *m, const double *u,
+                      uint32_t *active, uint32_t *tie);
+
+/* ---- S4 plant (P:242 delta-sigma, P:238/P:264 meter, Eq. 5, Eq. 8/10b) */
+void ora_plant_step(const ora_cfg *c, const double *a_true, double c_true, const double *thr_max,
+                    const double *dem, double noise, const double *u0, double *acc, double *fbar,
+                    double *p, double *thr, uint8_t *levels);
+
+/* ---- generator front-ends (exposed for the device-generator bit test) */
+uint64_t ora_gen_mix64(uint64_t z);
+void ora_gen_server(const ora_cfg *c, uint64_t server, double *a_true, double *c_true,
+                    double *thr_max, double *base, double *amp);
+double ora_gen_noise(const ora_cfg *c, uint64_t server, int64_t k);
+void ora_gen_demand(const ora_cfg *c, const ora_workload *w, uint64_t server, int64_t k, double *dem);
+double ora_gen_cap_base(const ora_cfg *c, const ora_workload *w, uint64_t server, int cap_idx);
+
+/* ---- closed loop (P:90-96 loop, P:196 receding horizon).  Instances are
+ * global ids inst = server * n_caps + cap.  Trace arrays are [periods][n_inst][...]
+ * (any may be NULL).  Returns 0 or a negative error. */
+int ora_simulate(const ora_cfg *c, const ora_workload *w, int n_inst, const int64_t *inst,
+                 const double *caps_override /* [periods][n_inst] or NULL */,
+                 double *tr_p /* p(k) seen at instant k */, double *tr_cap, double *tr_u /*[M][N]*/,
+                 uint32_t *tr_active /*[M]*/, uint32_t *tr_tie /*[M]*/, int8_t *tr_rank /*[N]*/,
+                 uint8_t *tr_levels /*[S][N]*/, double *tr_ahat /*[N]*/, double *tr_theta /*[N]*/,
+                 uint32_t *tr_status, double *final_p /*[n_inst]: p(K)*/, ora_summary *summ,
+                 double *A0_out /*[n_inst][N]*/, int use_definition_mode);
+
+/* ---- S5 hierarchical budget (cfg 4, Q16) */
+void ora_budget_caps(int n_servers, int rack, const double *pmin, const double *w, double W,
+                     double B_c, double pmin_tot, const double *B_rack_max, double *cap);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
