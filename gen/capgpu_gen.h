@@ -142,15 +142,26 @@ GEN_HD double gen_dem_amp(uint64_t seed, uint64_t server, int j) {
 /* Bursty demand of knob j in period k:
  *   dem = thr_max * clamp(base + amp*[U_burst(k/10) < 0.2] + 0.05*(2U_jit(k) - 1), 0, 1.5)
  * key_jit / key_burst = gen_stream_key(seed, GEN_TAG_JIT / GEN_TAG_BURST, server). */
-GEN_HD double gen_demand_bursty(uint64_t key_jit, uint64_t key_burst, int j, int64_t k,
-                                double thr_max, double base, double amp) {
-  double ub = gen_u52(gen_sample(key_burst, (uint64_t)j, (uint64_t)(k / GEN_BURST_HOLD)));
+/* burst flag of knob j in burst epoch e = floor(k / GEN_BURST_HOLD) */
+GEN_HD int gen_burst_flag(uint64_t key_burst, int j, int64_t epoch) {
+  return gen_u52(gen_sample(key_burst, (uint64_t)j, (uint64_t)epoch)) < 0.2;
+}
+
+/* demand given the burst flag of the period's epoch */
+GEN_HD double gen_demand_flag(uint64_t key_jit, int j, int64_t k, int burst, double thr_max,
+                              double base, double amp) {
   double uj = gen_u52(gen_sample(key_jit, (uint64_t)j, (uint64_t)k));
-  double x = ub < 0.2 ? GEN_ADD(base, amp) : base;
+  double x = burst ? GEN_ADD(base, amp) : base;
   double t = GEN_ADD(GEN_MUL(2.0, uj), -1.0);
   double y = GEN_ADD(x, GEN_MUL(0.05, t));
   y = y < 0.0 ? 0.0 : (y > 1.5 ? 1.5 : y);
   return GEN_MUL(thr_max, y);
+}
+
+GEN_HD double gen_demand_bursty(uint64_t key_jit, uint64_t key_burst, int j, int64_t k,
+                                double thr_max, double base, double amp) {
+  return gen_demand_flag(key_jit, j, k, gen_burst_flag(key_burst, j, k / GEN_BURST_HOLD), thr_max,
+                         base, amp);
 }
 
 /* Constant demand: dem = thr_max * frac */

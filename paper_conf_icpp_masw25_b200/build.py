@@ -1,0 +1,89 @@
+"""Build the CUDA C-ABI library libcapgpu.so in-tree (nvcc, sm_100a).
+
+    python -m paper_conf_icpp_masw25_b200.build [--force]
+
+Every translation unit is compiled with
+``-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo`` (parallel, one
+process per unit) and linked with a static CUDA runtime plus the NCCL that
+ships with torch (site-packages/nvidia/nccl).  The host side is compiled with
+``-ffp-contract=off`` so host-computed tables reproduce the oracle's formulas.
+"""
+from __future__ import annotations
+
+import concurrent.futures as cf
+import glob
+import os
+import subprocess
+import sys
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(PKG)
+CSRC = os.path.join(PKG, "csrc")
+BUILD = os.path.join(PKG, "_build")
+LIB = os.path.join(PKG, "libcapgpu.so")
+NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def nccl_dirs():
+    import importlib.util
+    spec = importlib.util.find_spec("nvidia")
+    cands = []
+    if spec and spec.submodule_search_locations:
+        for p in spec.submodule_search_locations:
+            cands.append(os.path.join(p, "nccl"))
+    cands.append("/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl")
+    for c in cands:
+        if os.path.exists(os.path.join(c, "include", "nccl.h")):
+            return os.path.join(c, "include"), os.path.join(c, "lib")
+    raise RuntimeError("nccl.h not found (torch's nvidia-nccl wheel)")
+
+
+def cflags():
+    inc, _ = nccl_dirs()
+    return [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-ffp-contract=off",
+            "-Xcompiler", "-fno-fast-math", f"-I{inc}", f"-I{os.path.join(ROOT, 'include')}",
+            f"-I{os.path.join(ROOT, 'gen')}"]
+
+
+def _deps():
+    return (glob.glob(os.path.join(CSRC, "*.cuh")) + [os.path.join(ROOT, "include", "capgpu.h"),
+                                                      os.path.join(ROOT, "gen", "capgpu_gen.h")])
+
+
+def _compile(src: str, force: bool, verbose: bool) -> str:
+    obj = os.path.join(BUILD, os.path.basename(src).replace(".cu", ".o"))
+    newest_dep = max(os.path.getmtime(d) for d in _deps() + [src])
+    if not force and os.path.exists(obj) and os.path.getmtime(obj) >= newest_dep:
+        return obj
+    cmd = [NVCC, *cflags(), "-c", src, "-o", obj]
+    if verbose:
+        cmd.insert(1, "-Xptxas=-v")
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr[-8000:]}")
+    if verbose:
+        with open(obj + ".ptxas.txt", "w") as fh:
+            fh.write(r.stderr)
+    return obj
+
+
+def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -> str:
+    os.makedirs(BUILD, exist_ok=True)
+    srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    jobs = jobs or max(1, min(len(srcs), os.cpu_count() or 4))
+    with cf.ThreadPoolExecutor(jobs) as ex:
+        objs = list(ex.map(lambda s: _compile(s, force, verbose), srcs))
+    newest = max(os.path.getmtime(o) for o in objs)
+    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < newest:
+        _, libdir = nccl_dirs()
+        cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-cudart", "static", f"-L{libdir}", "-l:libnccl.so.2",
+               "-Xlinker", f"-rpath,{libdir}"]
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"link failed:\n{r.stderr[-8000:]}")
+    return LIB
+
+
+if __name__ == "__main__":
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

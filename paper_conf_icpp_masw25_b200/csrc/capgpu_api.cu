@@ -1,0 +1,596 @@
+// capgpu_api.cu -- the C ABI of include/capgpu.h: validation, device state
+// ownership, dispatch to the per-N kernel instantiations.
+//
+// Nothing here computes the method on the host: every step (S0-S5) runs in the
+// kernels of capgpu_kernels.cuh.  Host code only validates, allocates, builds
+// the per-launch constant block (grid, bounds, horizon weights, capacity table)
+// and launches.
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "capgpu_kernels.cuh"
+#include "capgpu_budget.cuh"
+
+using namespace capgpu;
+
+struct capgpu_ctx {
+  int64_t n_srv = 0, n_inst = 0;
+  int32_t N = 0, M = 0, P = 0, T = 0;
+  capgpu_params prm{};
+  capgpu_shard shard{};
+  capgpu_knob_bounds bounds[CAPGPU_MAX_KNOBS]{};
+  DevParams dp{};
+  StatePtrs st{};
+  Launchers L{};
+  void *ws = nullptr;
+  int64_t ws_bytes = 0;
+  bool servers_ready = false, has_prior = false, sim_ready = false;
+  int64_t k_global = 0;
+  capgpu_workload wl{};
+  Budget budget{};
+  char err[512] = {0};
+};
+
+static thread_local char g_err[512];
+
+static int fail(capgpu_ctx *c, int code, const char *fmt, ...) {
+  char *buf = c ? c->err : g_err;
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, 512, fmt, ap);
+  va_end(ap);
+  return code;
+}
+
+static int cuda_fail(capgpu_ctx *c, cudaError_t e, const char *where) {
+  return fail(c, CAPGPU_E_CUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+#define CK_CUDA(ctx, call)                                   \
+  do {                                                       \
+    cudaError_t e_ = (call);                                 \
+    if (e_ != cudaSuccess) return cuda_fail(ctx, e_, #call); \
+  } while (0)
+
+static bool is_device_ptr(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+#define NEED_DEV(ctx, ptr)                                                                  \
+  do {                                                                                      \
+    if (!is_device_ptr(ptr)) return fail(ctx, CAPGPU_E_INVALID, "%s is not a device pointer", #ptr); \
+  } while (0)
+#define OPT_DEV(ctx, ptr)                        \
+  do {                                           \
+    if ((ptr) != nullptr) NEED_DEV(ctx, ptr);    \
+  } while (0)
+
+static Launchers launchers(int N, int M) {
+  switch (N) {
+    case 2: return launchers_n2(M);
+    case 3: return launchers_n3(M);
+    case 4: return launchers_n4(M);
+    case 5: return launchers_n5(M);
+    case 6: return launchers_n6(M);
+    case 7: return launchers_n7(M);
+    case 8: return launchers_n8(M);
+    case 9: return launchers_n9(M);
+    case 10: return launchers_n10(M);
+    case 11: return launchers_n11(M);
+    case 12: return launchers_n12(M);
+    case 13: return launchers_n13(M);
+    case 14: return launchers_n14(M);
+    case 15: return launchers_n15(M);
+    case 16: return launchers_n16(M);
+    default: return Launchers{};
+  }
+}
+
+extern "C" {
+
+const char *capgpu_version(void) { return "capgpu-b200 0.1 (sm_100a)"; }
+
+const char *capgpu_status_string(int code) {
+  switch (code) {
+    case CAPGPU_OK: return "ok";
+    case CAPGPU_E_INVALID: return "invalid argument";
+    case CAPGPU_E_NOMEM: return "out of device memory";
+    case CAPGPU_E_CUDA: return "CUDA error";
+    case CAPGPU_E_NCCL: return "NCCL error";
+    case CAPGPU_E_ORDER: return "call order (no prior / not initialised)";
+    case CAPGPU_E_UNSUPPORTED: return "unsupported by this build";
+    default: return "unknown";
+  }
+}
+
+const char *capgpu_last_error(const capgpu_ctx *ctx) { return ctx ? ctx->err : g_err; }
+
+void capgpu_default_params(capgpu_params *o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof *o);
+  o->q = 1.0;
+  o->r0 = 1e-4;
+  o->theta_min = 0.05;
+  o->lambda = 0.95;
+  o->rho = 100.0;
+  o->a_lo = 0.25;
+  o->a_hi = 4.0;
+  o->a_floor = 1e-3;
+  o->gamma = 0.91;
+  o->noise_std = 11.0;
+  o->substeps = 4;
+  o->caps_per_server = 1;
+  o->seed = 1;
+}
+
+int64_t capgpu_shard_range(int64_t n_global, int32_t world, int32_t rank, int64_t granule, int64_t *begin_out) {
+  if (n_global <= 0 || world <= 0 || rank < 0 || rank >= world || granule <= 0) return -1;
+  const int64_t units = (n_global + granule - 1) / granule;
+  const int64_t base = units / world, rem = units % world;
+  // the first (world - rem) ranks get `base` units, the last `rem` ranks base + 1
+  const int64_t lo_ranks = world - rem;
+  int64_t u0 = rank < lo_ranks ? rank * base : lo_ranks * base + (rank - lo_ranks) * (base + 1);
+  int64_t nu = rank < lo_ranks ? base : base + 1;
+  int64_t b = u0 * granule, e = (u0 + nu) * granule;
+  if (e > n_global) e = n_global;
+  if (b > n_global) b = n_global;
+  if (begin_out) *begin_out = b;
+  return e - b;
+}
+
+int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_horizons h,
+                  const capgpu_knob_bounds *bounds, const capgpu_params *params, const capgpu_shard *shard) {
+  if (!out) return fail(nullptr, CAPGPU_E_INVALID, "out is NULL");
+  *out = nullptr;
+  capgpu_params prm;
+  if (params) prm = *params;
+  else capgpu_default_params(&prm);
+  const int N = 1 + n_gpus;
+  if (n_servers < 1) return fail(nullptr, CAPGPU_E_INVALID, "n_servers < 1");
+  if (n_gpus < 1 || N > CAPGPU_MAX_KNOBS) return fail(nullptr, CAPGPU_E_INVALID, "n_gpus must be in [1, 15]");
+  if (h.M < 1 || h.M > h.P || h.P > CAPGPU_MAX_P) return fail(nullptr, CAPGPU_E_INVALID, "need 1 <= M <= P <= 64");
+  if (h.M > CAPGPU_MAX_M) return fail(nullptr, CAPGPU_E_UNSUPPORTED, "M > %d", CAPGPU_MAX_M);
+  if (!bounds) return fail(nullptr, CAPGPU_E_INVALID, "bounds is NULL");
+  if (!(prm.q > 0) || !(prm.r0 > 0) || !(prm.theta_min > 0 && prm.theta_min <= 1) ||
+      !(prm.lambda > 0 && prm.lambda <= 1) || !(prm.rho > 0) || !(prm.a_lo >= 0 && prm.a_lo <= prm.a_hi) ||
+      !(prm.a_floor > 0) || !(prm.gamma > 0) || !(prm.noise_std >= 0) || prm.caps_per_server < 1)
+    return fail(nullptr, CAPGPU_E_INVALID, "params out of range");
+  if (!(prm.substeps == 1 || prm.substeps == 2 || prm.substeps == 4 || prm.substeps == 8))
+    return fail(nullptr, CAPGPU_E_INVALID, "substeps must be 1, 2, 4 or 8");
+  for (int j = 0; j < N; ++j) {
+    const capgpu_knob_bounds &b = bounds[j];
+    if (!(b.f_min < b.f_max) || !std::isfinite(b.f_min) || !std::isfinite(b.f_max))
+      return fail(nullptr, CAPGPU_E_INVALID, "knob %d: need f_min < f_max", j);
+    if (b.n_levels < 2 || b.n_levels > CAPGPU_MAX_LEVELS)
+      return fail(nullptr, CAPGPU_E_INVALID, "knob %d: n_levels in [2, 32]", j);
+    if (b.sweep_base < 0 || b.sweep_base >= b.n_levels) return fail(nullptr, CAPGPU_E_INVALID, "knob %d: sweep_base", j);
+    const double flo = b.f_lo == 0.0 ? b.f_min : b.f_lo;
+    if (!(flo >= b.f_min && flo <= b.f_max)) return fail(nullptr, CAPGPU_E_INVALID, "knob %d: f_lo outside [f_min, f_max]", j);
+    if (b.r0 < 0) return fail(nullptr, CAPGPU_E_INVALID, "knob %d: r0 < 0", j);
+  }
+  capgpu_shard sh{};
+  if (shard) sh = *shard;
+  else {
+    sh.rank = 0;
+    sh.world = 1;
+    sh.srv_begin = 0;
+    sh.n_servers_global = n_servers;
+  }
+  if (sh.world < 1 || sh.rank < 0 || sh.rank >= sh.world || sh.srv_begin < 0)
+    return fail(nullptr, CAPGPU_E_INVALID, "bad shard");
+  if (sh.n_servers_global < sh.srv_begin + n_servers) sh.n_servers_global = sh.srv_begin + n_servers;
+
+  capgpu_ctx *c = new (std::nothrow) capgpu_ctx();
+  if (!c) return fail(nullptr, CAPGPU_E_NOMEM, "host allocation");
+  c->n_srv = n_servers;
+  c->n_inst = n_servers * prm.caps_per_server;
+  c->N = N;
+  c->M = h.M;
+  c->P = h.P;
+  c->T = N * (N + 1) / 2;
+  c->prm = prm;
+  c->shard = sh;
+  for (int j = 0; j < N; ++j) c->bounds[j] = bounds[j];
+  c->L = launchers(N, h.M);
+
+  // ---- per-launch constants
+  DevParams &d = c->dp;
+  d.N = N;
+  d.M = h.M;
+  d.P = h.P;
+  d.S = prm.substeps;
+  d.n_caps = prm.caps_per_server;
+  d.q = prm.q;
+  d.theta_min = prm.theta_min;
+  d.lam = prm.lambda;
+  d.rho = prm.rho;
+  d.a_lo = prm.a_lo;
+  d.a_hi = prm.a_hi;
+  d.a_floor = prm.a_floor;
+  d.noise_scale = prm.noise_std * std::sqrt(3.0);
+  d.inv_S = 1.0 / (double)prm.substeps;
+  // Q11: c_t = Q for t < M-1, c_{M-1} = (P - M + 1) Q
+  for (int t = 0; t < h.M; ++t) d.ct[t] = t < h.M - 1 ? prm.q : (double)(h.P - h.M + 1) * prm.q;
+  d.seed = prm.seed;
+  d.srv_begin = sh.srv_begin;
+  d.n_srv = c->n_srv;
+  d.n_inst = c->n_inst;
+  for (int j = 0; j < N; ++j) {
+    const capgpu_knob_bounds &b = bounds[j];
+    KnobConst &k = d.k[j];
+    k.f_min = b.f_min;
+    k.f_max = b.f_max;
+    k.L = b.n_levels;
+    k.sweep_base = b.sweep_base;
+    k.step = (b.f_max - b.f_min) / (double)(b.n_levels - 1);
+    k.inv_step = 1.0 / k.step;
+    k.lo = b.f_lo == 0.0 ? b.f_min : b.f_lo;
+    k.hi = b.f_max;
+    k.m = b.f_min;  // Q7
+    k.r0 = b.r0 == 0.0 ? prm.r0 : b.r0;
+    k.inv_r0 = 1.0 / k.r0;
+    for (int l = 0; l < CAPGPU_MAX_LEVELS; ++l) {
+      const double lv = b.f_min + (double)(l < b.n_levels ? l : b.n_levels - 1) * k.step;
+      d.g[j][l] = j == 0 ? lv / b.f_max : std::pow(lv / b.f_max, prm.gamma);  // Q14
+    }
+  }
+
+  // ---- state workspace (SoA)
+  const int64_t ni = c->n_inst, ns = c->n_srv;
+  const int64_t nd_inst = (int64_t)(5 * N + c->T + 4);
+  const int64_t nd_srv = (int64_t)(5 * N + 3);
+  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 4 * (int64_t)h.M * ni + 4 * ni + 256;
+  cudaError_t e = cudaMalloc(&c->ws, (size_t)bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return fail(nullptr, CAPGPU_E_NOMEM, "cudaMalloc(%lld): %s", (long long)bytes, cudaGetErrorString(e));
+  }
+  c->ws_bytes = bytes;
+  cudaMemset(c->ws, 0, (size_t)bytes);
+  double *q = (double *)c->ws;
+  auto take = [&](int64_t n) { double *r = q; q += n; return r; };
+  StatePtrs &s = c->st;
+  s.fbar = take(N * ni);
+  s.acc = take(N * ni);
+  s.thr = take(N * ni);
+  s.p = take(ni);
+  s.w = take(ni);
+  s.mu_f = take(N * ni);
+  s.mu_p = take(ni);
+  s.S = take(c->T * ni);
+  s.Sfp = take(N * ni);
+  s.cap_base = take(ni);
+  s.a_true = take(N * ns);
+  s.c_true = take(ns);
+  s.thr_max = take(N * ns);
+  s.base = take(N * ns);
+  s.amp = take(N * ns);
+  s.A0 = take(N * ns);
+  s.pmin = take(ns);
+  s.pmax = take(ns);
+  s.act = (uint32_t *)q;
+  s.trace_slot = (int32_t *)(s.act + (int64_t)h.M * ni);
+
+  if (sh.use_nccl) {
+    int rc = budget_init_nccl(c->budget, sh.nccl_id, sh.world, sh.rank, c->err);
+    if (rc != CAPGPU_OK) {
+      cudaFree(c->ws);
+      delete c;
+      return fail(nullptr, rc, "nccl init failed");
+    }
+  }
+  *out = c;
+  return CAPGPU_OK;
+}
+
+int capgpu_destroy(capgpu_ctx *c) {
+  if (!c) return CAPGPU_OK;
+  budget_free(c->budget);
+  if (c->ws) cudaFree(c->ws);
+  delete c;
+  return CAPGPU_OK;
+}
+
+int64_t capgpu_state_bytes(const capgpu_ctx *c) { return c ? c->ws_bytes : 0; }
+
+static int ensure_servers(capgpu_ctx *c, cudaStream_t s) {
+  if (c->servers_ready) return CAPGPU_OK;
+  int e = c->L.init_servers(c->dp, c->st, s);
+  if (e) return cuda_fail(c, (cudaError_t)e, "init_servers");
+  c->servers_ready = true;
+  return CAPGPU_OK;
+}
+
+int capgpu_identify(capgpu_ctx *c, const double *F_d, const double *p_d, int32_t rows, double *A_out_d,
+                    double *C_out_d, double *r2_out_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  cudaStream_t s = (cudaStream_t)stream;
+  if ((F_d == nullptr) != (p_d == nullptr)) return fail(c, CAPGPU_E_INVALID, "F_d and p_d must both be set or both NULL");
+  if (F_d) {
+    NEED_DEV(c, F_d);
+    NEED_DEV(c, p_d);
+    if (rows < c->N + 1) return fail(c, CAPGPU_E_INVALID, "rows < N + 1");
+  } else {
+    rows = 0;
+    for (int j = 0; j < c->N; ++j) rows += c->bounds[j].n_levels;
+  }
+  OPT_DEV(c, A_out_d);
+  OPT_DEV(c, C_out_d);
+  OPT_DEV(c, r2_out_d);
+  if (!F_d) {
+    int rc = ensure_servers(c, s);
+    if (rc) return rc;
+  }
+  int e = c->L.identify(c->dp, c->st, F_d, p_d, rows, A_out_d, C_out_d, r2_out_d, s);
+  if (e) return cuda_fail(c, (cudaError_t)e, "identify");
+  c->has_prior = true;
+  return CAPGPU_OK;
+}
+
+int capgpu_set_prior(capgpu_ctx *c, const double *A0_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, A0_d);
+  CK_CUDA(c, cudaMemcpyAsync(c->st.A0, A0_d, sizeof(double) * c->N * c->n_srv, cudaMemcpyDeviceToDevice,
+                             (cudaStream_t)stream));
+  c->has_prior = true;
+  return CAPGPU_OK;
+}
+
+int capgpu_model_reset(capgpu_ctx *c, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int64_t ni = c->n_inst;
+  CK_CUDA(c, cudaMemsetAsync(c->st.w, 0, sizeof(double) * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.mu_f, 0, sizeof(double) * c->N * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.mu_p, 0, sizeof(double) * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.S, 0, sizeof(double) * c->T * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.Sfp, 0, sizeof(double) * c->N * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.act, 0, sizeof(uint32_t) * c->M * ni, s));
+  return CAPGPU_OK;
+}
+
+int capgpu_assign_weights(capgpu_ctx *c, const double *thr_d, const double *thr_max_d, double *theta_out_d,
+                          double *R_out_d, int8_t *rank_out_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, thr_d);
+  NEED_DEV(c, thr_max_d);
+  OPT_DEV(c, theta_out_d);
+  OPT_DEV(c, R_out_d);
+  OPT_DEV(c, rank_out_d);
+  int e = c->L.assign_weights(c->dp, thr_d, thr_max_d, theta_out_d, R_out_d, rank_out_d, c->n_srv,
+                              (cudaStream_t)stream);
+  if (e) return cuda_fail(c, (cudaError_t)e, "assign_weights");
+  return CAPGPU_OK;
+}
+
+int capgpu_control_step(capgpu_ctx *c, const double *p_meas_d, const double *f_applied_d, const double *thr_d,
+                        const double *thr_max_d, const double *cap_d, double *u_out_d, uint32_t *active_out_d,
+                        int8_t *rank_out_d, double *ahat_out_d, uint32_t *status_out_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  if (c->prm.caps_per_server != 1) return fail(c, CAPGPU_E_INVALID, "control_step needs caps_per_server == 1");
+  NEED_DEV(c, p_meas_d);
+  NEED_DEV(c, f_applied_d);
+  NEED_DEV(c, thr_d);
+  NEED_DEV(c, thr_max_d);
+  NEED_DEV(c, cap_d);
+  NEED_DEV(c, u_out_d);
+  NEED_DEV(c, active_out_d);
+  OPT_DEV(c, rank_out_d);
+  OPT_DEV(c, ahat_out_d);
+  OPT_DEV(c, status_out_d);
+  if (!c->has_prior) return fail(c, CAPGPU_E_ORDER, "no prior A0: call capgpu_identify or capgpu_set_prior first");
+  int e = c->L.control_step(c->dp, c->st, p_meas_d, f_applied_d, thr_d, thr_max_d, cap_d, u_out_d, active_out_d,
+                            rank_out_d, ahat_out_d, status_out_d, (cudaStream_t)stream);
+  if (e) return cuda_fail(c, (cudaError_t)e, "control_step");
+  return CAPGPU_OK;
+}
+
+__global__ void k_trace_slots(int32_t *slot, int64_t n, const int64_t *inst, int32_t n_trace) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) slot[i] = -1;
+  __syncthreads();
+}
+__global__ void k_trace_slots_set(int32_t *slot, int64_t n, const int64_t *inst, int32_t n_trace) {
+  const int t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t < n_trace) {
+    const int64_t i = inst[t];
+    if (i >= 0 && i < n) slot[i] = t;
+  }
+}
+
+int capgpu_sim_reset(capgpu_ctx *c) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  c->sim_ready = false;
+  c->k_global = 0;
+  return CAPGPU_OK;
+}
+
+static void apply_workload(DevParams &d, const capgpu_workload &w) {
+  d.demand_kind = w.demand_kind;
+  d.demand_frac = w.demand_frac;
+  d.cap_frac0 = w.cap_frac0;
+  d.cap_frac_rand = w.cap_frac_rand;
+  d.cap_frac_step = w.cap_frac_step;
+  d.cap_period = w.cap_period;
+  d.cap_lo = w.cap_lo;
+  d.cap_hi = w.cap_hi;
+  d.cap_mult = w.cap_mult;
+}
+
+int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, const capgpu_trace *tr,
+                    void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  if (!wl) return fail(c, CAPGPU_E_INVALID, "workload is NULL");
+  if (periods < 1 || periods > (1ll << 30)) return fail(c, CAPGPU_E_INVALID, "periods out of range");
+  if (wl->demand_kind != 0 && wl->demand_kind != 1) return fail(c, CAPGPU_E_INVALID, "demand_kind");
+  if (wl->cap_period < 0 || (wl->cap_period > 0 && !(wl->cap_lo >= 0 && wl->cap_lo <= wl->cap_hi)))
+    return fail(c, CAPGPU_E_INVALID, "cap schedule");
+  if (wl->hierarchical && c->prm.caps_per_server != 1)
+    return fail(c, CAPGPU_E_INVALID, "hierarchical budget needs caps_per_server == 1");
+  TracePtrs t{};
+  if (tr) {
+    OPT_DEV(c, tr->sum_p_d);
+    OPT_DEV(c, tr->sumsq_p_d);
+    OPT_DEV(c, tr->max_p_d);
+    OPT_DEV(c, tr->sum_theta_d);
+    OPT_DEV(c, tr->n_viol_d);
+    OPT_DEV(c, tr->n_window_d);
+    OPT_DEV(c, tr->act_count_d);
+    OPT_DEV(c, tr->final_p_d);
+    if (tr->n_trace < 0) return fail(c, CAPGPU_E_INVALID, "n_trace < 0");
+    if (tr->n_trace > 0) {
+      NEED_DEV(c, tr->trace_inst_d);
+      OPT_DEV(c, tr->p_d);
+      OPT_DEV(c, tr->cap_d);
+      OPT_DEV(c, tr->u_d);
+      OPT_DEV(c, tr->ahat_d);
+      OPT_DEV(c, tr->theta_d);
+      OPT_DEV(c, tr->active_d);
+      OPT_DEV(c, tr->rank_d);
+      OPT_DEV(c, tr->levels_d);
+      OPT_DEV(c, tr->status_d);
+      if (periods > (1ll << 24)) return fail(c, CAPGPU_E_INVALID, "traced runs are limited to 2^24 periods");
+    }
+    OPT_DEV(c, tr->agg_W_d);
+    OPT_DEV(c, tr->agg_P_d);
+    t.sum_p = tr->sum_p_d;
+    t.sumsq_p = tr->sumsq_p_d;
+    t.max_p = tr->max_p_d;
+    t.sum_theta = tr->sum_theta_d;
+    t.final_p = tr->final_p_d;
+    t.n_viol = tr->n_viol_d;
+    t.n_window = tr->n_window_d;
+    t.act_count = tr->act_count_d;
+    t.n_trace = tr->n_trace;
+    t.p = tr->p_d;
+    t.cap = tr->cap_d;
+    t.u = tr->u_d;
+    t.ahat = tr->ahat_d;
+    t.theta = tr->theta_d;
+    t.active = tr->active_d;
+    t.status = tr->status_d;
+    t.rank = tr->rank_d;
+    t.levels = tr->levels_d;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  apply_workload(c->dp, *wl);
+  if (!c->sim_ready) {
+    int rc = ensure_servers(c, s);
+    if (rc) return rc;
+    int rows = 0;
+    for (int j = 0; j < c->N; ++j) rows += c->bounds[j].n_levels;
+    int e = c->L.identify(c->dp, c->st, nullptr, nullptr, rows, nullptr, nullptr, nullptr, s);
+    if (e) return cuda_fail(c, (cudaError_t)e, "identify (simulate init)");
+    c->has_prior = true;
+    e = c->L.init_instances(c->dp, c->st, s);
+    if (e) return cuda_fail(c, (cudaError_t)e, "init_instances");
+    c->sim_ready = true;
+    c->k_global = 0;
+    c->wl = *wl;
+    if (wl->hierarchical) {
+      int rb = budget_setup(c->budget, c->dp, c->st, *wl, c->shard, s, c->err);
+      if (rb) return rb;
+    }
+  }
+  if (t.n_trace > 0) {
+    k_trace_slots<<<grid_for(c->n_inst, 256), 256, 0, s>>>(c->st.trace_slot, c->n_inst, nullptr, 0);
+    k_trace_slots_set<<<grid_for(t.n_trace, 256), 256, 0, s>>>(c->st.trace_slot, c->n_inst, tr->trace_inst_d,
+                                                               t.n_trace);
+    CK_CUDA(c, cudaGetLastError());
+  }
+  if (wl->hierarchical) {
+    int rc = budget_simulate(c->budget, c->dp, c->st, t, c->L, c->k_global, periods, tr ? tr->agg_W_d : nullptr,
+                             tr ? tr->agg_P_d : nullptr, s, c->err);
+    if (rc) return rc;
+  } else {
+    int e = c->L.simulate(c->dp, c->st, t, c->k_global, (int)periods, s);
+    if (e) return cuda_fail(c, (cudaError_t)e, "simulate");
+  }
+  c->k_global += periods;
+  return CAPGPU_OK;
+}
+
+int capgpu_sim_state(capgpu_ctx *c, double *fbar_d, double *acc_d, double *thr_d, double *p_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  OPT_DEV(c, fbar_d);
+  OPT_DEV(c, acc_d);
+  OPT_DEV(c, thr_d);
+  OPT_DEV(c, p_d);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t nb = sizeof(double) * c->N * c->n_inst;
+  if (fbar_d) CK_CUDA(c, cudaMemcpyAsync(fbar_d, c->st.fbar, nb, cudaMemcpyDeviceToDevice, s));
+  if (acc_d) CK_CUDA(c, cudaMemcpyAsync(acc_d, c->st.acc, nb, cudaMemcpyDeviceToDevice, s));
+  if (thr_d) CK_CUDA(c, cudaMemcpyAsync(thr_d, c->st.thr, nb, cudaMemcpyDeviceToDevice, s));
+  if (p_d) CK_CUDA(c, cudaMemcpyAsync(p_d, c->st.p, sizeof(double) * c->n_inst, cudaMemcpyDeviceToDevice, s));
+  return CAPGPU_OK;
+}
+
+int capgpu_debug_gen(capgpu_ctx *c, int64_t k, int32_t demand_kind, double demand_frac, double *a_true_d,
+                     double *thr_max_d, double *c_true_d, double *dem_d, double *noise_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, a_true_d);
+  NEED_DEV(c, thr_max_d);
+  NEED_DEV(c, c_true_d);
+  NEED_DEV(c, dem_d);
+  NEED_DEV(c, noise_d);
+  DevParams d = c->dp;
+  d.demand_kind = demand_kind;
+  d.demand_frac = demand_frac;
+  int e = c->L.debug_gen(d, c->st, k, a_true_d, thr_max_d, c_true_d, dem_d, noise_d, (cudaStream_t)stream);
+  if (e) return cuda_fail(c, (cudaError_t)e, "debug_gen");
+  return CAPGPU_OK;
+}
+
+// FP64 pipe microbenchmark: 8 independent DFMA chains per thread.
+__global__ void k_dfma_peak(double *out, int iters, double a, double b) {
+  double x[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = threadIdx.x * 1e-3 + c;
+  for (int i = 0; i < iters; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) x[c] = fma(x[c], a, b);
+  }
+  double s = 0;
+#pragma unroll
+  for (int c = 0; c < 8; ++c) s += x[c];
+  if (s == 12345.678) out[0] = s;
+}
+
+int capgpu_fp64_peak(double *tflops_out, void *stream) {
+  if (!tflops_out) return fail(nullptr, CAPGPU_E_INVALID, "out is NULL");
+  cudaStream_t s = (cudaStream_t)stream;
+  int dev = 0, sms = 0;
+  CK_CUDA(nullptr, cudaGetDevice(&dev));
+  CK_CUDA(nullptr, cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  double *d = nullptr;
+  CK_CUDA(nullptr, cudaMalloc(&d, 64));
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  const int blocks = sms * 4, thr = 256, iters = 1 << 14;
+  k_dfma_peak<<<blocks, thr, 0, s>>>(d, 64, 1.0000001, 1e-9);
+  cudaEventRecord(e0, s);
+  for (int r = 0; r < 5; ++r) k_dfma_peak<<<blocks, thr, 0, s>>>(d, iters, 1.0000001, 1e-9);
+  cudaEventRecord(e1, s);
+  cudaError_t e = cudaEventSynchronize(e1);
+  float ms = 0;
+  cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFree(d);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "fp64 peak");
+  *tflops_out = 5.0 * blocks * thr * (double)iters * 8 * 2 / (ms * 1e-3) / 1e12;
+  return CAPGPU_OK;
+}
+
+}  // extern "C"
