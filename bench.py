@@ -1,0 +1,320 @@
+#!/usr/bin/env python
+"""Benchmark of the CapGPU hot path on B200: server-control-steps/s.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--periods P]
+    python bench.py --impl reference ...        # the CPU oracle as the reference arm
+
+One bench "step" = one call of the public C ABI `capgpu_simulate` advancing
+every instance of the workload by `--periods` control periods (default: the
+config's run length), i.e. (instances x periods) server-control-steps, all of
+S1-S4 per step.  Default workload: BASELINE.json configs[2]
+(cfg 3: 65,536 servers, 1 CPU + 8 GPUs, P/M = 8/3, 1,000 periods, bursty
+demand and throughput-driven weights) - see DESIGN.md §8 for why cfg 3.
+
+Timing: W untimed warm-up steps, then K timed steps, each bracketed by CUDA
+events on the launching stream; L2 is flushed (256 MiB write) between timed
+steps outside the events; barrier + synchronize on both sides; max over ranks.
+Multi-GPU (torchrun): one process per GPU, weak scaling (each rank runs its own
+disjoint shard of the config, no data-path collective).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from gen import configs  # noqa: E402
+
+B200_SMS = 148
+FP64_FMA_PER_CLK_PER_SM = 64          # DFMA lanes per SM (measured: 34.1 TF = 92 % of 37.2 at 1965 MHz)
+SM_MAX_MHZ = 1965.0
+
+
+def algorithmic_flops(N: int, M: int, S: int) -> float:
+    """Algorithmic FP64 work per server-control-step, div/sqrt = 1."""
+    model = 2 + 4 * (N + 1) + 3 * N * (N + 1) / 2 + 6 * N + N ** 3 / 3 + 2 * N ** 2
+    mpc = 3 * N + 2 + 18 * M * N
+    plant = 4 * N * S + 7 * N + 6
+    return model + mpc + plant + (5 * N + M + 1)
+
+
+def state_bytes_per_instance(N: int, M: int) -> int:
+    T = N * (N + 1) // 2
+    return 8 * 2 * (5 * N + T + 4) + 4 * 2 * M  # read + write once per call (fused mode)
+
+
+def fp64_peak_derived() -> float:
+    return B200_SMS * FP64_FMA_PER_CLK_PER_SM * 2 * SM_MAX_MHZ * 1e6 / 1e12
+
+
+# ---------------------------------------------------------------- clocks
+
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+           0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+           0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+class ClockSampler(threading.Thread):
+    def __init__(self, index: int, period_s: float = 0.02):
+        super().__init__(daemon=True)
+        self.samples, self.period, self.stop_evt, self.ok = [], period_s, threading.Event(), False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+
+    def run(self):
+        if not self.ok:
+            return
+        nv = self.nv
+        get_r = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or nv.nvmlDeviceGetCurrentClocksThrottleReasons
+        while not self.stop_evt.is_set():
+            try:
+                self.samples.append((time.monotonic(), nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM),
+                                     int(get_r(self.h))))
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def summary(self, t0: float, t1: float):
+        self.stop_evt.set()
+        win = [s for s in self.samples if t0 <= s[0] <= t1] or self.samples[-5:]
+        if not win:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"], "samples": 0}
+        bits = 0
+        for s in win:
+            bits |= s[2]
+        reasons = [n for b, n in REASONS.items() if bits & b and n != "gpu_idle"]
+        return {"sm_mhz": statistics.median(s[1] for s in win), "sm_max_mhz": self.max_mhz, "reasons": reasons,
+                "samples": len(win)}
+
+
+# ---------------------------------------------------------------- oracle (CPU baseline / reference arm)
+
+def _oracle_worker(args):
+    cfg, insts, periods = args
+    from oracle import oracle as O
+    o = O.oracle_for(cfg)
+    t = time.perf_counter()
+    o.simulate(insts, periods=periods, traces=False)
+    return time.perf_counter() - t
+
+
+def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int):
+    """Oracle (as it stands) on `cores` host processes over a bounded sample of
+    the workload; returns (steps/s, sample description, cores)."""
+    import multiprocessing as mp
+    from oracle import oracle as O
+    O.build()
+    desc = configs.get(cfg)
+    n_inst = desc["n_servers"] * desc["workload"]["n_caps"]
+    cal_p = min(periods, 100)
+    t_cal = _oracle_worker((cfg, [0], cal_p))
+    per_inst = t_cal / cal_p * periods
+    k = max(1, int(budget_s / max(per_inst, 1e-6)))
+    stride = max(1, n_inst // (k * cores))
+    jobs = [(cfg, [((w * k + i) * stride) % n_inst for i in range(k)], periods) for w in range(cores)]
+    ctx = mp.get_context("fork")
+    t0 = time.perf_counter()
+    with ctx.Pool(cores) as pool:
+        pool.map(_oracle_worker, jobs)
+    wall = time.perf_counter() - t0
+    steps = cores * k * periods
+    return steps / wall, f"{cores * k} instances (strided over the {n_inst}) x {periods} periods", cores, wall
+
+
+# ---------------------------------------------------------------- main
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3, 5])
+    ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
+    ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle work for cpu_baseline")
+    return ap.parse_args()
+
+
+def workload_name(d, periods):
+    return (f"cfg{d['cfg']}: {d['n_servers']:,} servers x {d['workload']['n_caps']} caps, 1 CPU + "
+            f"{d['n_gpus']} GPUs (N={d['n_gpus'] + 1}), P/M={d['P']}/{d['M']}, {periods} periods per step")
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    d = configs.get(args.config)
+    periods = args.periods or d["periods"]
+    cores = os.cpu_count() or 1
+    total_steps, total_t = 0.0, 0.0
+    budget = max(1.0, 60.0 / max(1, args.steps + args.warmup))
+    for it in range(args.warmup + args.steps):
+        rate, sample, cores_used, wall = oracle_rate(args.config, periods, budget, cores)
+        if it >= args.warmup:
+            total_steps += rate * wall
+            total_t += wall
+    value = total_steps / total_t
+    N = d["n_gpus"] + 1
+    line = {"impl": "reference", "metric": "server-control-steps/sec", "value": value,
+            "unit": "server-control-steps/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * total_t / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded, DESIGN.md §3)",
+            "config": {"workload": workload_name(d, periods), "n_knobs": N, "P": d["P"], "M": d["M"]},
+            "cpu_baseline": {"value": value, "unit": "server-control-steps/s", "cores": cores_used,
+                             "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "server-control-steps/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_masw25_b200 import CapGPU, workload_from
+    from paper_conf_icpp_masw25_b200 import capgpu as G
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    d = configs.get(args.config)
+    periods = args.periods or d["periods"]
+    n_srv = d["n_servers"]
+    N, M, S = d["n_gpus"] + 1, d["M"], d["controller"]["substeps"]
+    g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=rank * n_srv, world=world, rank=rank,
+                           n_servers_global=world * n_srv)
+    wl = workload_from(d)
+    n_inst = g.n_inst
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+        torch.cuda.synchronize()
+
+    # warm-up (includes the one-time identification sweep + init)
+    bufs = g.summary_buffers()
+    for _ in range(args.warmup):
+        g.simulate(periods, wl, out=bufs)
+    barrier()
+
+    sampler = ClockSampler(local)
+    sampler.start()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    barrier()
+    t0 = time.monotonic()
+    for i in range(args.steps):
+        flush.zero_()  # L2 flush outside the timed events
+        evs[i][0].record(stream)
+        g.simulate(periods, wl, out=bufs)
+        evs[i][1].record(stream)
+    barrier()
+    t1 = time.monotonic()
+    clocks = sampler.summary(t0, t1)
+    ms = [a.elapsed_time(b) for a, b in evs]
+    t_local = sum(ms) / 1e3
+    tt = torch.tensor([t_local], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    t_max = float(tt.item())
+    steps_per_call = n_inst * periods
+    value = world * steps_per_call * args.steps / t_max
+
+    # ---- e2e through the public API with host buffers: H2D of the per-instance
+    # set points from pinned memory, capgpu_simulate, D2H of the summaries.
+    caps_host = g.sim_caps().cpu().pin_memory()
+    caps_dev = torch.empty_like(caps_host, device=dev)
+    outs_host = {k: torch.empty(n_inst, dtype=dt, pin_memory=True)
+                 for k, dt in (("sum_p", torch.float64), ("max_p", torch.float64), ("n_viol", torch.int32))}
+    e2e_evs = []
+    for i in range(max(3, args.steps // 2)):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        caps_dev.copy_(caps_host, non_blocking=True)
+        wl.cap_base_d = caps_dev.data_ptr()
+        out = g.simulate(periods, wl, out=bufs)
+        for k in outs_host:
+            outs_host[k].copy_(out[k], non_blocking=True)
+        b.record(stream)
+        e2e_evs.append((a, b))
+    wl.cap_base_d = None
+    barrier()
+    t_e2e = sum(a.elapsed_time(b) for a, b in e2e_evs) / 1e3
+    te = torch.tensor([t_e2e], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_value = world * steps_per_call * len(e2e_evs) / float(te.item())
+
+    flops = algorithmic_flops(N, M, S)
+    launch_s = t_local / args.steps
+    achieved = flops * steps_per_call / launch_s / 1e12
+    peak = fp64_peak_derived()
+    measured_peak = G.fp64_peak_tflops()
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}_summary.json")
+    if os.path.exists(prof):
+        try:
+            pj = json.load(open(prof))
+            if pj.get("periods") == periods and pj.get("n_inst") == n_inst:
+                traffic = pj.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    if rank == 0:
+        line = {"metric": "server-control-steps/sec", "value": value, "unit": "server-control-steps/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": 1e3 * t_max / args.steps, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded generator, DESIGN.md §3)",
+                "config": {"workload": workload_name(d, periods), "instances_per_gpu": n_inst,
+                           "periods_per_step": periods, "n_knobs": N, "P": d["P"], "M": M, "substeps": S,
+                           "mode": "fused multi-period kernel k_simulate (1 launch per step)",
+                           "l2": "flushed between timed steps (256 MiB write outside the events)",
+                           "parallelism": f"dp{world} (server shards, no data-path collective)"},
+                "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                             "frac": achieved / peak, "traffic": traffic,
+                             "flops_per_step": flops,
+                             "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 x 1965 MHz "
+                                            "(DESIGN.md §8); measured DFMA microbench in peak_measured",
+                             "peak_measured": measured_peak,
+                             "state_bytes_per_step": state_bytes_per_instance(N, M) / periods},
+                "e2e": {"value": e2e_value, "unit": "server-control-steps/s", "h2d_bytes_per_step": 8 * n_inst,
+                        "d2h_bytes_per_step": 20 * n_inst},
+                "gpu_launches": args.steps,
+                "clocks": clocks}
+        if world == 1 and not args.no_cpu_baseline:
+            rate, sample, cores, _ = oracle_rate(args.config, periods, args.cpu_budget, os.cpu_count() or 1)
+            line["cpu_baseline"] = {"value": rate, "unit": "server-control-steps/s", "cores": cores,
+                                    "kind": "oracle", "sample": sample}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -147,15 +147,27 @@ GEN_HD int gen_burst_flag(uint64_t key_burst, int j, int64_t epoch) {
   return gen_u52(gen_sample(key_burst, (uint64_t)j, (uint64_t)epoch)) < 0.2;
 }
 
-/* demand given the burst flag of the period's epoch */
-GEN_HD double gen_demand_flag(uint64_t key_jit, int j, int64_t k, int burst, double thr_max,
-                              double base, double amp) {
-  double uj = gen_u52(gen_sample(key_jit, (uint64_t)j, (uint64_t)k));
+/* jitter uniform of knob j in period k: knobs 2q and 2q+1 share one hash
+ * (26-bit halves), so a server draws ceil(N/2) jitter hashes per period */
+GEN_HD uint64_t gen_jit_hash(uint64_t key_jit, int pair, int64_t k) {
+  return gen_sample(key_jit, (uint64_t)pair, (uint64_t)k);
+}
+GEN_HD double gen_jit_u(uint64_t h, int j) { return (j & 1) ? gen_u26_lo(h) : gen_u26_hi(h); }
+
+/* demand from the jitter uniform and the burst flag:
+ * thr_max * clamp(base + amp*burst + 0.05 (2u - 1), 0, 1.5) */
+GEN_HD double gen_demand_u(double uj, int burst, double thr_max, double base, double amp) {
   double x = burst ? GEN_ADD(base, amp) : base;
   double t = GEN_ADD(GEN_MUL(2.0, uj), -1.0);
   double y = GEN_ADD(x, GEN_MUL(0.05, t));
   y = y < 0.0 ? 0.0 : (y > 1.5 ? 1.5 : y);
   return GEN_MUL(thr_max, y);
+}
+
+/* demand given the burst flag of the period's epoch */
+GEN_HD double gen_demand_flag(uint64_t key_jit, int j, int64_t k, int burst, double thr_max,
+                              double base, double amp) {
+  return gen_demand_u(gen_jit_u(gen_jit_hash(key_jit, j >> 1, k), j), burst, thr_max, base, amp);
 }
 
 GEN_HD double gen_demand_bursty(uint64_t key_jit, uint64_t key_burst, int j, int64_t k,

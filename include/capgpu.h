@@ -111,6 +111,8 @@ typedef struct {
   int32_t block;             /* servers per reduction block (1024) */
   double cluster_frac;       /* B_c = Pmin_tot + cluster_frac (Pmax_tot - Pmin_tot) */
   double rack_frac;          /* B_rack = rack_frac * sum_rack Pmax */
+  const double *cap_base_d;  /* nullable device [n_inst]: operator-set base caps P_s (W) for this
+                                call, replacing the generated ones (the step schedule still applies) */
 } capgpu_workload;
 
 /* Optional outputs of capgpu_simulate; every pointer may be NULL.
@@ -210,6 +212,10 @@ int capgpu_sim_reset(capgpu_ctx *ctx);
  * (device pointers, nullable). */
 int capgpu_sim_state(capgpu_ctx *ctx, double *fbar_d, double *acc_d, double *thr_d, double *p_d,
                      void *stream);
+
+/* Current base caps P_s of every local instance (device [n_inst], W); valid
+ * after the first capgpu_simulate. */
+int capgpu_sim_caps(capgpu_ctx *ctx, double *cap_base_d, void *stream);
 
 /* Multi-GPU helper: ncclUniqueId (128 bytes) to broadcast from rank 0. */
 int capgpu_nccl_unique_id(uint8_t out[128]);

@@ -24,6 +24,9 @@ OK, E_INVALID, E_NOMEM, E_CUDA, E_NCCL, E_ORDER, E_UNSUPPORTED = 0, -1, -2, -3, 
 ST_CAP_INFEASIBLE, ST_SLO_INFEASIBLE, ST_SOLVER_CAP, ST_NONFINITE = 1, 2, 4, 8
 
 
+_VP = C.c_void_p
+
+
 class Horizons(C.Structure):
     _fields_ = [("P", C.c_int32), ("M", C.c_int32)]
 
@@ -50,7 +53,7 @@ class Workload(C.Structure):
                 ("cap_frac_rand", C.c_double), ("cap_frac_step", C.c_double), ("cap_period", C.c_int64),
                 ("cap_lo", C.c_int64), ("cap_hi", C.c_int64), ("cap_mult", C.c_double),
                 ("hierarchical", C.c_int32), ("rack", C.c_int32), ("block", C.c_int32),
-                ("cluster_frac", C.c_double), ("rack_frac", C.c_double)]
+                ("cluster_frac", C.c_double), ("rack_frac", C.c_double), ("cap_base_d", _VP)]
 
 
 _VP = C.c_void_p
@@ -67,7 +70,7 @@ class Trace(C.Structure):
 SYMBOLS = ["capgpu_version", "capgpu_status_string", "capgpu_last_error", "capgpu_default_params",
            "capgpu_create", "capgpu_destroy", "capgpu_state_bytes", "capgpu_identify", "capgpu_set_prior",
            "capgpu_model_reset", "capgpu_assign_weights", "capgpu_control_step", "capgpu_simulate",
-           "capgpu_sim_reset", "capgpu_sim_state", "capgpu_nccl_unique_id", "capgpu_shard_range",
+           "capgpu_sim_reset", "capgpu_sim_state", "capgpu_sim_caps", "capgpu_nccl_unique_id", "capgpu_shard_range",
            "capgpu_debug_gen", "capgpu_fp64_peak"]
 
 _lib = None
@@ -101,6 +104,7 @@ def lib():
     L.capgpu_simulate.argtypes = [_VP, C.c_int64, C.POINTER(Workload), C.POINTER(Trace), _VP]
     L.capgpu_sim_reset.argtypes = [_VP]
     L.capgpu_sim_state.argtypes = [_VP, _VP, _VP, _VP, _VP, _VP]
+    L.capgpu_sim_caps.argtypes = [_VP, _VP, _VP]
     L.capgpu_nccl_unique_id.argtypes = [C.POINTER(C.c_uint8 * 128)]
     L.capgpu_shard_range.argtypes = [C.c_int64, C.c_int32, C.c_int32, C.c_int64, C.POINTER(C.c_int64)]
     L.capgpu_shard_range.restype = C.c_int64
@@ -264,15 +268,20 @@ class CapGPU:
         return dict(u=u, active=act, rank=rk, ahat=ah, status=st)
 
     # ---- closed loop
+    def summary_buffers(self):
+        """Per-instance summary outputs (written entirely by the kernel; reusable)."""
+        ni, M = self.n_inst, self.M
+        e = lambda *s, dtype=torch.float64: torch.empty(*s, dtype=dtype, device=self.device)  # noqa: E731
+        return dict(sum_p=e(ni), sumsq_p=e(ni), max_p=e(ni), sum_theta=e(ni), n_viol=e(ni, dtype=torch.int32),
+                    n_window=e(ni, dtype=torch.int32), act_count=e(M, ni, dtype=torch.int32), final_p=e(ni))
+
     def simulate(self, periods: int, workload: Workload, trace_inst=None, summaries: bool = True,
-                 traces=("p", "cap", "u", "ahat", "theta", "active", "rank", "levels", "status")):
+                 traces=("p", "cap", "u", "ahat", "theta", "active", "rank", "levels", "status"), out=None):
         ni, N, M, S = self.n_inst, self.N, self.M, self.S
         tr = Trace()
-        out = {}
+        if out is None:
+            out = self.summary_buffers() if summaries else {}
         if summaries:
-            out.update(sum_p=self._z(ni), sumsq_p=self._z(ni), max_p=self._z(ni), sum_theta=self._z(ni),
-                       n_viol=self._z(ni, dtype=torch.int32), n_window=self._z(ni, dtype=torch.int32),
-                       act_count=self._z(M, ni, dtype=torch.int32), final_p=self._z(ni))
             for k in ("sum_p", "sumsq_p", "max_p", "sum_theta", "n_viol", "n_window", "act_count", "final_p"):
                 setattr(tr, k + "_d", _ptr(out[k]).value)
         if trace_inst is not None:
@@ -305,6 +314,11 @@ class CapGPU:
         f, a, t, p = self._z(N, ni), self._z(N, ni), self._z(N, ni), self._z(ni)
         _check(self.L.capgpu_sim_state(self._ctx, _ptr(f), _ptr(a), _ptr(t), _ptr(p), _stream()), self._ctx)
         return dict(fbar=f, acc=a, thr=t, p=p)
+
+    def sim_caps(self):
+        out = self._z(self.n_inst)
+        _check(self.L.capgpu_sim_caps(self._ctx, _ptr(out), _stream()), self._ctx)
+        return out
 
     def debug_gen(self, k: int, demand_kind: int = 1, demand_frac: float = 0.7):
         n, N = self.n_srv, self.N

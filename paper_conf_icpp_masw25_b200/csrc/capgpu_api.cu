@@ -224,6 +224,39 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   d.srv_begin = sh.srv_begin;
   d.n_srv = c->n_srv;
   d.n_inst = c->n_inst;
+  d.inv_N = 1.0 / (double)N;
+  // Frequency-grid classes: knobs with the same (f_min, f_max, L, CPU/GPU)
+  // share one table of thresholds, levels and capacity factors (Q14, Q15),
+  // computed here with the oracle's formulas (host, no FP contraction).
+  static_assert(sizeof(GridEntry) == 32, "GridEntry layout");
+  GridEntry grid[CAPGPU_MAX_KNOBS][CAPGPU_MAX_LEVELS];
+  int n_class = 0;
+  int cls_of[CAPGPU_MAX_KNOBS];
+  for (int j = 0; j < N; ++j) {
+    const capgpu_knob_bounds &b = bounds[j];
+    int found = -1;
+    for (int q = 0; q < j; ++q) {
+      const capgpu_knob_bounds &o = bounds[q];
+      if (o.f_min == b.f_min && o.f_max == b.f_max && o.n_levels == b.n_levels && (q == 0) == (j == 0)) {
+        found = cls_of[q];
+        break;
+      }
+    }
+    if (found < 0) {
+      found = n_class++;
+      const double step = (b.f_max - b.f_min) / (double)(b.n_levels - 1);
+      for (int l = 0; l < CAPGPU_MAX_LEVELS; ++l) {
+        GridEntry &e = grid[found][l];
+        const int ll = l < b.n_levels ? l : b.n_levels - 1;
+        e.level = b.f_min + (double)ll * step;
+        e.g = j == 0 ? e.level / b.f_max : std::pow(e.level / b.f_max, prm.gamma);  // Q14
+        e.mid_lo = ll == 0 ? -INFINITY : b.f_min + ((double)(ll - 1) + 0.5) * step;
+        e.mid_hi = ll >= b.n_levels - 1 ? INFINITY : b.f_min + ((double)ll + 0.5) * step;
+      }
+    }
+    cls_of[j] = found;
+  }
+  d.n_class = n_class;
   for (int j = 0; j < N; ++j) {
     const capgpu_knob_bounds &b = bounds[j];
     KnobConst &k = d.k[j];
@@ -231,6 +264,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     k.f_max = b.f_max;
     k.L = b.n_levels;
     k.sweep_base = b.sweep_base;
+    k.cls = cls_of[j];
     k.step = (b.f_max - b.f_min) / (double)(b.n_levels - 1);
     k.inv_step = 1.0 / k.step;
     k.lo = b.f_lo == 0.0 ? b.f_min : b.f_lo;
@@ -238,17 +272,17 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     k.m = b.f_min;  // Q7
     k.r0 = b.r0 == 0.0 ? prm.r0 : b.r0;
     k.inv_r0 = 1.0 / k.r0;
-    for (int l = 0; l < CAPGPU_MAX_LEVELS; ++l) {
-      const double lv = b.f_min + (double)(l < b.n_levels ? l : b.n_levels - 1) * k.step;
-      d.g[j][l] = j == 0 ? lv / b.f_max : std::pow(lv / b.f_max, prm.gamma);  // Q14
-    }
   }
+  d.convex = 1;
+  for (int j = 0; j < N; ++j) d.convex &= d.k[j].lo == d.k[j].m ? 1 : 0;
 
   // ---- state workspace (SoA)
   const int64_t ni = c->n_inst, ns = c->n_srv;
   const int64_t nd_inst = (int64_t)(5 * N + c->T + 4);
   const int64_t nd_srv = (int64_t)(5 * N + 3);
-  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 4 * (int64_t)h.M * ni + 4 * ni + 256;
+  const int64_t grid_bytes = (int64_t)sizeof(GridEntry) * n_class * CAPGPU_MAX_LEVELS;
+  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 8 * (int64_t)h.M * ni + 4 * ni + grid_bytes +
+                        (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 256;
   cudaError_t e = cudaMalloc(&c->ws, (size_t)bytes);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -278,8 +312,16 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   s.A0 = take(N * ns);
   s.pmin = take(ns);
   s.pmax = take(ns);
-  s.act = (uint32_t *)q;
-  s.trace_slot = (int32_t *)(s.act + (int64_t)h.M * ni);
+  s.s_prev = take((int64_t)h.M * ni);
+  GridEntry *gdev = (GridEntry *)take(4 * (int64_t)n_class * CAPGPU_MAX_LEVELS);
+  KnobConst *kdev = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 7) / 8);
+  cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice);
+  d.k_dev = kdev;
+  s.trace_slot = (int32_t *)q;
+  for (int c2 = 0; c2 < n_class; ++c2)
+    cudaMemcpy(gdev + c2 * CAPGPU_MAX_LEVELS, grid[c2], sizeof(GridEntry) * CAPGPU_MAX_LEVELS,
+               cudaMemcpyHostToDevice);
+  d.grid = gdev;
 
   if (sh.use_nccl) {
     int rc = budget_init_nccl(c->budget, sh.nccl_id, sh.world, sh.rank, c->err);
@@ -355,7 +397,7 @@ int capgpu_model_reset(capgpu_ctx *c, void *stream) {
   CK_CUDA(c, cudaMemsetAsync(c->st.mu_p, 0, sizeof(double) * ni, s));
   CK_CUDA(c, cudaMemsetAsync(c->st.S, 0, sizeof(double) * c->T * ni, s));
   CK_CUDA(c, cudaMemsetAsync(c->st.Sfp, 0, sizeof(double) * c->N * ni, s));
-  CK_CUDA(c, cudaMemsetAsync(c->st.act, 0, sizeof(uint32_t) * c->M * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.s_prev, 0, sizeof(double) * c->M * ni, s));
   return CAPGPU_OK;
 }
 
@@ -502,6 +544,11 @@ int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, c
       if (rb) return rb;
     }
   }
+  if (wl->cap_base_d) {
+    NEED_DEV(c, wl->cap_base_d);
+    CK_CUDA(c, cudaMemcpyAsync(c->st.cap_base, wl->cap_base_d, sizeof(double) * c->n_inst,
+                               cudaMemcpyDeviceToDevice, s));
+  }
   if (t.n_trace > 0) {
     k_trace_slots<<<grid_for(c->n_inst, 256), 256, 0, s>>>(c->st.trace_slot, c->n_inst, nullptr, 0);
     k_trace_slots_set<<<grid_for(t.n_trace, 256), 256, 0, s>>>(c->st.trace_slot, c->n_inst, tr->trace_inst_d,
@@ -532,6 +579,15 @@ int capgpu_sim_state(capgpu_ctx *c, double *fbar_d, double *acc_d, double *thr_d
   if (acc_d) CK_CUDA(c, cudaMemcpyAsync(acc_d, c->st.acc, nb, cudaMemcpyDeviceToDevice, s));
   if (thr_d) CK_CUDA(c, cudaMemcpyAsync(thr_d, c->st.thr, nb, cudaMemcpyDeviceToDevice, s));
   if (p_d) CK_CUDA(c, cudaMemcpyAsync(p_d, c->st.p, sizeof(double) * c->n_inst, cudaMemcpyDeviceToDevice, s));
+  return CAPGPU_OK;
+}
+
+int capgpu_sim_caps(capgpu_ctx *c, double *cap_base_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, cap_base_d);
+  if (!c->sim_ready) return fail(c, CAPGPU_E_ORDER, "simulation not initialised");
+  CK_CUDA(c, cudaMemcpyAsync(cap_base_d, c->st.cap_base, sizeof(double) * c->n_inst, cudaMemcpyDeviceToDevice,
+                             (cudaStream_t)stream));
   return CAPGPU_OK;
 }
 

@@ -1,10 +1,18 @@
-// capgpu_device.cuh -- per-server device math of the CapGPU step (sm_100a, FP64).
+// capgpu_device.cuh -- per-instance device math of the CapGPU step (sm_100a, FP64).
 //
 // One CUDA thread owns one (server, cap) instance.  All loops over knobs are
-// compile-time (template N) and fully unrolled, so the per-server model,
-// Hessian factors and QP state live in registers; the symmetric scatter
-// Sigma_ff and the read-only per-server constants live in a per-thread
-// shared-memory slab (SoA [field][thread], conflict-free 8-byte accesses).
+// compile-time (template N) and fully unrolled, so the model, its LDL^T
+// factors and the QP state live in registers.
+//
+// Instruction economy (the kernel is FP64-pipe / issue bound):
+//   - clamps are plain compare+select (no fmin/fmax NaN handling), sums
+//     are split in two partial accumulators for ILP;
+//   - rarely executed code (QP phase 2, trace replays) is out of line so the
+//     hot period loop fits the instruction cache;
+//   - divisions that only feed continuous values use an MUFU seed + 2 Newton
+//     steps; the one division that decides integers (theta -> ranks) is IEEE;
+//   - frequency-grid arithmetic that must match the oracle bit for bit comes
+//     from host-computed tables staged in shared memory.
 //
 // Citations: P:NNN = PAPER.md line; Qn = DESIGN.md §2 reading.
 #pragma once
@@ -31,32 +39,43 @@ struct Tri {
   }
 };
 
-// Uniform (per-launch) constants.  Passed by value as the kernel parameter
-// (constant bank); the level-capacity table is staged into shared memory.
+// Uniform (per-launch) constants, passed by value (constant bank).
 struct KnobConst {
   double f_min, f_max, step, inv_step;  // grid (Q15)
   double lo, hi, m;                     // box [l, h] (Eq. 10a, Q14) and penalty reference f_min (Q7)
   double r0, inv_r0;                    // r0_j and 1 / r0_j (Q6, Q9)
   int32_t L;                            // levels
   int32_t sweep_base;
+  int32_t cls;                          // grid class (knobs with identical grids share a table)
+  int32_t pad;
+};
+
+// Per-class grid table entry, level l:  {mid(l-1) or -inf, mid(l) or +inf,
+// level(l), g(l)}: decision thresholds, frequency and capacity factor (Q14, Q15).
+struct GridEntry {
+  double mid_lo, mid_hi, level, g;
 };
 
 struct DevParams {
   int32_t N, M, P, S;
   int32_t n_caps;            // instances per server
   int32_t demand_kind;
+  int32_t n_class;
+  int32_t convex;            // 1 iff lo_j == m_j (= f_min) for every knob: phi convex on s <= 0
   double demand_frac;
   double q, theta_min, lam, rho, a_lo, a_hi, a_floor;
   double noise_scale;        // sigma * sqrt(3) (host-computed)
   double inv_S;              // 1/S, exact (S power of two, Q22)
+  double inv_N;              // 1/N for the mean-theta summary
   double ct[kMaxM];          // block weights c_t (Q11)
   double cap_frac0, cap_frac_rand, cap_frac_step, cap_mult;
   int64_t cap_period, cap_lo, cap_hi;
   uint64_t seed;
   int64_t srv_begin;         // global id of local server 0
   int64_t n_srv, n_inst;     // local counts
+  const GridEntry *grid;     // device [n_class][kMaxL]
+  const KnobConst *k_dev;    // device copy of k[] for out-of-line code (keeps P in the param bank)
   KnobConst k[kMaxN];
-  double g[kMaxN][kMaxL];    // capacity factor g_j(l) (Q14)
 };
 
 // ------------------------------------------------------------------ helpers
@@ -71,41 +90,30 @@ __device__ __forceinline__ double rcp_fast(double x) {
   return fma(y, e, y);
 }
 
-__device__ __forceinline__ double clampd(double x, double lo, double hi) { return fmin(fmax(x, lo), hi); }
+__device__ __forceinline__ long long dbits(double x) { return __double_as_longlong(x); }
+__device__ __forceinline__ double bitsd(long long b) { return __longlong_as_double(b); }
 
-// Exact level arithmetic (Q15): must reproduce the host formulas bit for bit,
-// so no FMA contraction here.
-__device__ __forceinline__ double level_value(const KnobConst &kc, int l) {
-  return __dadd_rn(kc.f_min, __dmul_rn((double)l, kc.step));
-}
-__device__ __forceinline__ double level_mid(const KnobConst &kc, int l) {
-  return __dadd_rn(kc.f_min, __dmul_rn((double)l + 0.5, kc.step));
-}
-// #{midpoints < v}: estimate from the grid, then one exact correction each way.
-__device__ __forceinline__ int level_index(const KnobConst &kc, double v) {
-  double x = fma(v - kc.f_min, kc.inv_step, 0.5);
-  int l = __double2int_rd(x);
-  l = min(max(l, 0), kc.L - 1);
-  if (l > 0 && v <= level_mid(kc, l - 1)) --l;
-  else if (l < kc.L - 1 && v > level_mid(kc, l)) ++l;
-  return l;
+// clamp without fmin/fmax NaN handling: one DSETP + two FSEL per side
+__device__ __forceinline__ double pclamp(double x, double lo, double hi) {
+  return x < lo ? lo : (x > hi ? hi : x);
 }
 
 // ------------------------------------------------------------------ S1 model
 // Weighted Welford push (Q1-Q3): w <- lam w + 1, delta = z - mu,
 // mu += delta / w, Sigma <- lam Sigma + (1 - 1/w) delta delta^T
 // (= delta (z - mu_new)^T in exact arithmetic).
-template <int N, class SAcc>
-__device__ __forceinline__ void model_push(double lam, double &w, double (&mu_f)[N], double &mu_p,
-                                           SAcc S, double (&Sfp)[N], const double (&f)[N], double p) {
+template <int N, class SAcc, class VAcc>
+__device__ __forceinline__ void model_push(double lam, double &w, VAcc mu_f, double &mu_p, SAcc S, VAcc Sfp,
+                                           const double (&f)[N], double p) {
   w = fma(lam, w, 1.0);
   const double iw = rcp_fast(w);
   const double e = 1.0 - iw;
   double df[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    df[j] = f[j] - mu_f[j];
-    mu_f[j] = fma(df[j], iw, mu_f[j]);
+    const double m = mu_f.get(j);
+    df[j] = f[j] - m;
+    mu_f.set(j, fma(df[j], iw, m));
   }
   const double dp = p - mu_p;
   mu_p = fma(dp, iw, mu_p);
@@ -118,7 +126,7 @@ __device__ __forceinline__ void model_push(double lam, double &w, double (&mu_f)
       const int t = Tri<N>::idx(i, j);
       S.set(t, fma(lam, S.get(t), ei * df[j]));
     }
-    Sfp[i] = fma(lam, Sfp[i], df[i] * edp);
+    Sfp.set(i, fma(lam, Sfp.get(i), df[i] * edp));
   }
 }
 
@@ -165,9 +173,9 @@ __device__ __forceinline__ void ldlt_solve(double (&L)[Tri<N>::size], const doub
 }
 
 // (Sigma_ff + rho I) a = Sigma_fp + rho A0, then clamp to [a_lo A0, a_hi A0] (Q1, Q4).
-template <int N, class SAcc, class A0Acc>
-__device__ __forceinline__ void model_solve(double rho, double a_lo, double a_hi, SAcc S,
-                                            const double (&Sfp)[N], A0Acc A0, double (&ahat)[N]) {
+template <int N, class SAcc, class VAcc, class A0Acc>
+__device__ __forceinline__ void model_solve(double rho, double a_lo, double a_hi, SAcc S, VAcc Sfp, A0Acc A0,
+                                            double (&ahat)[N]) {
   double L[Tri<N>::size];
 #pragma unroll
   for (int t = 0; t < Tri<N>::size; ++t) L[t] = S.get(t);
@@ -175,12 +183,12 @@ __device__ __forceinline__ void model_solve(double rho, double a_lo, double a_hi
   for (int j = 0; j < N; ++j) L[Tri<N>::idx(j, j)] += rho;
   double b[N];
 #pragma unroll
-  for (int i = 0; i < N; ++i) b[i] = fma(rho, A0.get(i), Sfp[i]);
+  for (int i = 0; i < N; ++i) b[i] = fma(rho, A0.get(i), Sfp.get(i));
   ldlt_solve<N>(L, b, ahat);
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     const double a0 = A0.get(j);
-    ahat[j] = clampd(ahat[j], a_lo * a0, a_hi * a0);
+    ahat[j] = pclamp(ahat[j], a_lo * a0, a_hi * a0);
   }
 }
 
@@ -191,7 +199,7 @@ template <int N>
 __device__ __forceinline__ void weights(double theta_min, const double (&thr)[N], const double (&thr_max)[N],
                                         double (&theta)[N]) {
 #pragma unroll
-  for (int j = 0; j < N; ++j) theta[j] = clampd(__ddiv_rn(thr[j], thr_max[j]), theta_min, 1.0);
+  for (int j = 0; j < N; ++j) theta[j] = pclamp(__ddiv_rn(thr[j], thr_max[j]), theta_min, 1.0);
 }
 
 template <int N>
@@ -202,7 +210,8 @@ __device__ __forceinline__ void ranks(const double (&theta)[N], int8_t (&rk)[N])
 #pragma unroll
     for (int l = 0; l < N; ++l) {
       if (l == j) continue;
-      r += (theta[l] > theta[j]) || (l < j && theta[l] == theta[j]);
+      const long long tl = dbits(theta[l]), tj = dbits(theta[j]);
+      r += (tl > tj) || (l < j && tl == tj);
     }
     rk[j] = (int8_t)r;
   }
@@ -212,134 +221,251 @@ __device__ __forceinline__ void ranks(const double (&theta)[N], int8_t (&rk)[N])
 // Block t of the decoupled Eq. 9 (Q11):
 //   min_{lo<=u<=hi} c (beta + a.u)^2 + sum_j R_j (u_j - m_j)^2
 // KKT: u_j(s) = clamp(m_j - c tau_j s, lo_j, hi_j), tau_j = a_j / R_j, and
-// s = beta + a.u(s).  phi(s) = s - beta - a.u(s) is strictly increasing and
-// piecewise linear (slope >= 1, breakpoints where a knob meets a bound), so
-// the root is unique and is the exact root of the linear piece it lies on.
-//   phase 1: up to 3 Newton steps on phi from the warm-start active set (the
-//            previous period's); ends when a Newton point reproduces its own
-//            active set (then it is the exact root).
+// s = beta + a.u(s) (the predicted tracking error).  phi(s) = s - beta - a.u(s)
+// is strictly increasing and piecewise linear with slope
+// phi'(s) = 1 + sum_{free j} c tau_j a_j >= 1, so the root is unique and is the
+// exact root of the linear piece it lies on.
+//   phase 1: Newton from the previous period's root s_prev (warm start):
+//            s' = s - phi(s)/phi'(s).  When the active set at s' equals the one
+//            at s, s' is the root of that piece: exact.  Two tries.
 //   phase 2: otherwise the root's active set is read off phi at each knob's
-//            two breakpoints (<= 2N evaluations, no sorting) and the root of
-//            that piece is exact.  Bounded work, no iteration cap to hit.
+//            two breakpoints (phi increasing: s* > b <=> phi(b) < 0; <= 2N
+//            evaluations, no sorting) and the root of that piece is exact.
 
-// root of the linear piece with active codes `code`
+// phi, slope and active codes at s.  cta_j = c tau_j a_j.  Per knob: one
+// DFMA for v, two DSETP, predicated accumulation (no selects on the FP64
+// pipe beyond the clamp).  Two partial sums for ILP.
 template <int N>
-__device__ __forceinline__ double piece_root(const KnobConst *kc, const double (&a)[N], const double (&ctau)[N],
-                                             double beta, uint32_t code) {
-  double num = beta, den = 1.0;
+__device__ __forceinline__ uint32_t block_eval(const KnobConst *kc, const double (&a)[N], const double (&ctau)[N],
+                                               const double (&cta)[N], double beta, double s, double &phi,
+                                               double &slope) {
+  uint32_t code = 0u;
+  double f0 = s - beta, f1 = 0.0, d0 = 1.0, d1 = 0.0;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    const uint32_t cj = (code >> (2 * j)) & 3u;
-    const double x = cj == 0u ? kc[j].m : (cj == 1u ? kc[j].lo : kc[j].hi);
-    num = fma(a[j], x, num);
-    den = cj == 0u ? fma(ctau[j], a[j], den) : den;
+    const double v = fma(-ctau[j], s, kc[j].m);
+    const bool low = v < kc[j].lo, up = v > kc[j].hi;
+    code |= (low ? 1u : 0u) << (2 * j);
+    code |= (up ? 2u : 0u) << (2 * j);
+    const double u = low ? kc[j].lo : (up ? kc[j].hi : v);
+    if (j & 1) {
+      f1 = fma(-a[j], u, f1);
+      if (!(low || up)) d1 += cta[j];
+    } else {
+      f0 = fma(-a[j], u, f0);
+      if (!(low || up)) d0 += cta[j];
+    }
+  }
+  phi = f0 + f1;
+  slope = d0 + d1;
+  return code;
+}
+
+template <int N>
+__device__ __forceinline__ uint32_t block_codes(const KnobConst *kc, const double (&ctau)[N], double s) {
+  uint32_t code = 0u;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    const double v = fma(-ctau[j], s, kc[j].m);
+    code |= (v < kc[j].lo ? 1u : 0u) << (2 * j);
+    code |= (v > kc[j].hi ? 2u : 0u) << (2 * j);
+  }
+  return code;
+}
+
+// phase 2 (rare): exact active set of the root read off phi at each knob's
+// breakpoints.  Kept out of line so the hot loop stays small (I-cache).
+template <int N>
+__device__ __noinline__ double block_exact(const KnobConst *kc, const double *a_p, const double *ctau_p,
+                                           double beta) {
+  double a[N], ctau[N], cta[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    a[j] = a_p[j];
+    ctau[j] = ctau_p[j];
+    cta[j] = ctau[j] * a[j];
+  }
+  double num = beta, den = 1.0;
+#pragma unroll 1
+  for (int j = 0; j < N; ++j) {
+    double x;
+    const double cj = ctau_p[j];
+    if (!(cj > 0.0)) {
+      x = pclamp(kc[j].m, kc[j].lo, kc[j].hi);
+    } else {
+      const double r = rcp_fast(cj);
+      double fb, sl;
+      block_eval<N>(kc, a, ctau, cta, beta, (kc[j].m - kc[j].lo) * r, fb, sl);
+      if (fb < 0.0) {
+        x = kc[j].lo;  // root right of b_l: lower
+      } else {
+        block_eval<N>(kc, a, ctau, cta, beta, (kc[j].m - kc[j].hi) * r, fb, sl);
+        if (fb > 0.0) {
+          x = kc[j].hi;  // root left of b_h: upper
+        } else {
+          x = kc[j].m;  // free
+          den += cj * a_p[j];
+        }
+      }
+    }
+    num = fma(a_p[j], x, num);
   }
   return num * rcp_fast(den);
 }
 
-// active codes and phi at s
+// Convex case (no SLO-raised lower bound: lo_j == m_j for all j).  For s >= 0
+// every knob sits at lo, so phi(s) = s - beta - a.lo there; for s < 0 each
+// u_j(s) = min(m_j - c tau_j s, hi_j) and phi is convex.  Hence:
+//   phi(0) <= 0  ->  s* = beta + a.lo >= 0 exactly (all knobs at lo);
+//   otherwise Newton from the right of the root converges monotonically (a
+//   start left of the root overshoots once to the right), each step landing
+//   on the root of the current piece; it ends when the new point stays in
+//   the piece (exact).  At most N + 2 steps, no safeguard needed.
+// a_lo_sum = sum_j a_j lo_j (shared by the blocks of an instant).
 template <int N>
-__device__ __forceinline__ uint32_t eval_phi(const KnobConst *kc, const double (&a)[N], const double (&ctau)[N],
-                                             double beta, double s, double &phi) {
-  uint32_t nc = 0u;
-  double f = s - beta;
+__device__ __forceinline__ double solve_block_convex(const KnobConst *kc, const double (&a)[N],
+                                                     const double (&ctau)[N], double beta, double a_lo_sum,
+                                                     double s_warm) {
+  const double phi0 = -(beta + a_lo_sum);
+  if (!(phi0 > 0.0)) return beta + a_lo_sum;
+  double cta[N], sum_cta = 1.0;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    const double v = fma(-ctau[j], s, kc[j].m);
-    const uint32_t cj = v < kc[j].lo ? 1u : (v > kc[j].hi ? 2u : 0u);
-    nc |= cj << (2 * j);
-    f = fma(-a[j], clampd(v, kc[j].lo, kc[j].hi), f);
+    cta[j] = ctau[j] * a[j];
+    sum_cta += cta[j];
   }
-  phi = f;
-  return nc;
+  double s, phi, slope;
+  uint32_t code;
+  if (s_warm < 0.0) {
+    s = s_warm;
+    code = block_eval<N>(kc, a, ctau, cta, beta, s, phi, slope);
+  } else {  // just left of 0: every knob free
+    s = 0.0;
+    phi = phi0;
+    slope = sum_cta;
+    code = 0u;
+  }
+#pragma unroll 1
+  for (int it = 0; it < N + 2; ++it) {
+    if (phi == 0.0) return s;
+    double s1 = fma(-phi, rcp_fast(slope), s);
+    if (s1 >= 0.0) {  // overshoot from the left: restart just left of 0
+      s1 = -phi0 * rcp_fast(sum_cta);
+      code = 0u;
+    }
+    if (block_codes<N>(kc, ctau, s1) == code) return s1;
+    s = s1;
+    code = block_eval<N>(kc, a, ctau, cta, beta, s, phi, slope);
+  }
+  return s;
 }
 
+// Solve one block; returns the root s (u and codes follow from it).
 template <int N>
-__device__ __forceinline__ uint32_t solve_block(const KnobConst *kc, const double (&a)[N],
-                                                const double (&tau)[N], double c, double beta,
-                                                uint32_t code, double (&u)[N], bool &capped) {
-  double ctau[N];
+__device__ __forceinline__ double solve_block(const KnobConst *kc, const KnobConst *kc_dev, const double (&a)[N],
+                                              const double (&ctau)[N],
+                                              double beta, double s_warm) {
+  double cta[N];
 #pragma unroll
-  for (int j = 0; j < N; ++j) ctau[j] = c * tau[j];
-  double s = 0.0;
-  bool done = false;
-  // phase 1: a few Newton steps from the warm start (the common case ends in
-  // the first: last period's active set is still right).
-  constexpr int kNewton = 3;
+  for (int j = 0; j < N; ++j) cta[j] = ctau[j] * a[j];
+  double s = s_warm;
 #pragma unroll 1
-  for (int it = 0; it < kNewton; ++it) {
-    s = piece_root<N>(kc, a, ctau, beta, code);
-    double phi;
-    const uint32_t nc = eval_phi<N>(kc, a, ctau, beta, s, phi);
-    if (nc == code || phi == 0.0) { done = true; break; }
-    code = nc;
+  for (int it = 0; it < 2; ++it) {
+    double phi, slope;
+    const uint32_t c0 = block_eval<N>(kc, a, ctau, cta, beta, s, phi, slope);
+    if (phi == 0.0) return s;
+    const double s1 = fma(-phi, rcp_fast(slope), s);
+    if (block_codes<N>(kc, ctau, s1) == c0) return s1;
+    s = s1;
   }
-  if (!done) {
-    // phase 2: the active set of the root read off phi at each knob's own
-    // breakpoints (phi increasing: s* > b  <=>  phi(b) < 0), no sorting:
-    //   lower  iff s* > b_l = (m - lo)/(c tau),  upper iff s* < b_h = (m - hi)/(c tau).
-    code = 0u;
+  double a_l[N], c_l[N];
 #pragma unroll
-    for (int j = 0; j < N; ++j) {
-      uint32_t cj;
-      if (!(ctau[j] > 0.0)) {
-        cj = kc[j].m < kc[j].lo ? 1u : (kc[j].m > kc[j].hi ? 2u : 0u);
-      } else {
-        const double r = rcp_fast(ctau[j]);
-        double fb;
-        eval_phi<N>(kc, a, ctau, beta, (kc[j].m - kc[j].lo) * r, fb);
-        if (fb < 0.0) {
-          cj = 1u;
-        } else {
-          eval_phi<N>(kc, a, ctau, beta, (kc[j].m - kc[j].hi) * r, fb);
-          cj = fb > 0.0 ? 2u : 0u;
-        }
-      }
-      code |= cj << (2 * j);
-    }
-    s = piece_root<N>(kc, a, ctau, beta, code);
-    // consistency: the classification at s must reproduce `code` (exact root);
-    // a mismatch can only come from a rounding-level tie and is reported.
-    double phi;
-    if (eval_phi<N>(kc, a, ctau, beta, s, phi) != code && fabs(phi) > 1e-9 * (1.0 + fabs(beta))) capped = true;
+  for (int j = 0; j < N; ++j) {
+    a_l[j] = a[j];
+    c_l[j] = ctau[j];
   }
-  uint32_t out = 0u;
+  return block_exact<N>(kc_dev, a_l, c_l, beta);
+}
+
+// u(s) and the 2-bit codes at the root (Q19: exact tie counts as free).
+template <int N>
+__device__ __forceinline__ uint32_t block_u(const KnobConst *kc, const double (&ctau)[N], double s, double (&u)[N]) {
+  uint32_t code = 0u;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     const double v = fma(-ctau[j], s, kc[j].m);
-    const uint32_t cj = v < kc[j].lo ? 1u : (v > kc[j].hi ? 2u : 0u);
-    out |= cj << (2 * j);
-    u[j] = clampd(v, kc[j].lo, kc[j].hi);
+    const bool low = v < kc[j].lo, up = v > kc[j].hi;
+    code |= (low ? 1u : 0u) << (2 * j);
+    code |= (up ? 2u : 0u) << (2 * j);
+    u[j] = low ? kc[j].lo : (up ? kc[j].hi : v);
   }
-  return out;
+  return code;
 }
 
 // ------------------------------------------------------------------ S4 plant
 // First-order delta-sigma over S sub-steps, period averages (Q22),
-// throughput min(dem, thr_max g(l)) (Q18).  Exact arithmetic (no contraction)
-// so level indices, fbar and thr reproduce the oracle bit for bit given u0.
+// throughput min(dem, thr_max g(l)) (Q18).  Exact arithmetic (no contraction;
+// thresholds, levels and capacities from the host tables) so level indices,
+// fbar and thr reproduce the oracle bit for bit given u0.  Sub-step loop
+// outside (not unrolled: small code), knobs inside (unrolled: ILP across
+// knobs).  grid = shared-memory copy of the per-class tables.
 template <int N>
-__device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const double *sg /* smem [N][kMaxL] */,
-                                                  const double (&u0)[N], double (&acc)[N],
-                                                  const double (&dem)[N], const double (&thr_max)[N],
-                                                  double (&fbar)[N], double (&thr)[N], uint8_t *lv_out,
-                                                  int lv_stride) {
+__device__ __forceinline__ int level_of(const KnobConst &kc, const GridEntry *tab, double v) {
+  // estimate, then one exact correction each way against the thresholds
+  int l = __double2int_rd(fma(v - kc.f_min, kc.inv_step, 0.5));
+  l = min(max(l, 0), kc.L - 1);
+  const double2 mm = *reinterpret_cast<const double2 *>(&tab[l].mid_lo);
+  return l + (v > mm.y ? 1 : 0) - (v <= mm.x ? 1 : 0);
+}
+
+template <int N>
+__device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const GridEntry *grid, const double (&u0)[N],
+                                                  double (&acc)[N], const double (&dem)[N],
+                                                  const double (&thr_max)[N], double (&fbar)[N], double (&thr)[N]) {
+  double fs[N], ts[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    const KnobConst &kc = P.k[j];
-    double fs = 0.0, ts = 0.0, ac = acc[j];
-    for (int s = 0; s < P.S; ++s) {
-      const double v = __dadd_rn(u0[j], ac);
-      const int l = level_index(kc, v);
-      const double lv = level_value(kc, l);
-      ac = __dadd_rn(v, -lv);
-      fs = __dadd_rn(fs, lv);
-      ts = __dadd_rn(ts, fmin(dem[j], __dmul_rn(thr_max[j], sg[j * kMaxL + l])));
-      if (lv_out) lv_out[(s * N + j) * lv_stride] = (uint8_t)l;
+    fs[j] = 0.0;
+    ts[j] = 0.0;
+  }
+#pragma unroll 1
+  for (int s = 0; s < P.S; ++s) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const KnobConst &kc = P.k[j];
+      const GridEntry *tab = grid + kc.cls * kMaxL;
+      const double v = __dadd_rn(u0[j], acc[j]);
+      const int l = level_of<N>(kc, tab, v);
+      const double2 lg = *reinterpret_cast<const double2 *>(&tab[l].level);
+      acc[j] = __dadd_rn(v, -lg.x);
+      fs[j] = __dadd_rn(fs[j], lg.x);
+      const double capj = __dmul_rn(thr_max[j], lg.y);
+      ts[j] = __dadd_rn(ts[j], dem[j] < capj ? dem[j] : capj);
     }
-    acc[j] = ac;
-    fbar[j] = __dmul_rn(fs, P.inv_S);
-    thr[j] = __dmul_rn(ts, P.inv_S);
+  }
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    fbar[j] = __dmul_rn(fs[j], P.inv_S);
+    thr[j] = __dmul_rn(ts[j], P.inv_S);
+  }
+}
+
+// Trace of the level indices (traced instances only): replays the same
+// delta-sigma from the pre-period accumulators.  Out of line (I-cache).
+template <int N>
+__device__ __noinline__ void plant_trace_levels(const KnobConst *k_dev, int S, const GridEntry *grid,
+                                                const double *u0, const double *acc_in, uint8_t *lv_out,
+                                                int64_t lv_stride) {
+  for (int j = 0; j < N; ++j) {
+    const KnobConst &kc = k_dev[j];
+    const GridEntry *tab = grid + kc.cls * kMaxL;
+    double ac = acc_in[j];
+    for (int s = 0; s < S; ++s) {
+      const double v = __dadd_rn(u0[j], ac);
+      const int l = level_of<N>(kc, tab, v);
+      ac = __dadd_rn(v, -tab[l].level);
+      lv_out[(int64_t)(s * N + j) * lv_stride] = (uint8_t)l;
+    }
   }
 }
 

@@ -7,11 +7,12 @@
 //   k_init_instances cap base + virtual period -1 (Q23)
 //   k_simulate       S1-S4 fused over K periods, one THREAD per instance, state
 //                    in registers + a per-thread shared-memory slab
-//   k_period         S1-S4 for one period with state in HBM + rack/cluster
-//                    budget (S5, cfg 4)
+//   k_period         S1-S4 for one period with state in HBM (hierarchical budget)
 //   k_control_step   S1-S3 on user measurements (per-period mode)
 //   k_assign_weights S2 alone
 #pragma once
+
+#include <cmath>
 
 #include "capgpu_device.cuh"
 
@@ -24,7 +25,7 @@ struct StatePtrs {
   // per instance (ld = n_inst)
   double *fbar, *acc, *thr, *p;            // plant state S4
   double *w, *mu_f, *mu_p, *S, *Sfp;       // model state S1
-  uint32_t *act;                           // [M] warm-start active codes
+  double *s_prev;                          // [M] warm-start roots of the block QPs
   double *cap_base;                        // [1]
   int32_t *trace_slot;                     // [1] -1 = not traced
   // per server (ld = n_srv)
@@ -41,17 +42,19 @@ struct TracePtrs {
   uint8_t *levels;
 };
 
-struct SlabAcc {
+// per-thread slab in shared memory, AoS with an odd field count F: lane i
+// accesses 8-byte words at stride F -> conflict-free, compile-time offsets.
+struct Slab {
   double *p;
-  int stride;
-  __device__ __forceinline__ double get(int t) const { return p[t * stride]; }
-  __device__ __forceinline__ void set(int t, double v) const { p[t * stride] = v; }
+  __device__ __forceinline__ double get(int t) const { return p[t]; }
+  __device__ __forceinline__ void set(int t, double v) const { p[t] = v; }
 };
 
 template <int N>
 struct RegArr {
   double (&r)[N];
   __device__ __forceinline__ double get(int t) const { return r[t]; }
+  __device__ __forceinline__ void set(int t, double v) const { r[t] = v; }
 };
 
 // global-memory accessor for the per-period kernels (state in HBM)
@@ -62,10 +65,42 @@ struct GlobAcc {
   __device__ __forceinline__ void set(int t, double v) const { p[(int64_t)t * ld] = v; }
 };
 
-__device__ __forceinline__ double plant_power(double c_true, const double *a, const double *f, int n, double noise) {
-  double pw = c_true;
-  for (int j = 0; j < n; ++j) pw = fma(a[j], f[j], pw);
-  return pw + noise;
+__device__ __forceinline__ void load_grid(const DevParams &P, GridEntry *sgrid) {
+  const int n = P.n_class * kMaxL;
+  for (int t = threadIdx.x; t < n; t += blockDim.x) sgrid[t] = P.grid[t];
+}
+
+// ------------------------------------------------------------------ synthetic inputs (gen/capgpu_gen.h)
+
+template <int N>
+__device__ __forceinline__ uint32_t burst_mask(const DevParams &P, uint64_t kburst, int64_t epoch) {
+  uint32_t m = 0u;
+  if (P.demand_kind != 0) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) m |= (uint32_t)gen_burst_flag(kburst, j, epoch) << j;
+  }
+  return m;
+}
+
+// demand of all knobs in period k: one jitter hash per knob pair
+template <int N, class BaseAcc, class AmpAcc>
+__device__ __forceinline__ void demand_all(const DevParams &P, uint64_t kjit, int64_t k, uint32_t bmask,
+                                           const double (&thr_max)[N], BaseAcc base, AmpAcc amp,
+                                           double (&dem)[N]) {
+  if (P.demand_kind == 0) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) dem[j] = gen_demand_const(thr_max[j], P.demand_frac);
+    return;
+  }
+#pragma unroll
+  for (int q = 0; q < (N + 1) / 2; ++q) {
+    const uint64_t h = gen_jit_hash(kjit, q, k);
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int j = 2 * q + e;
+      if (j < N) dem[j] = gen_demand_u(gen_jit_u(h, j), (bmask >> j) & 1u, thr_max[j], base.get(j), amp.get(j));
+    }
+  }
 }
 
 // ------------------------------------------------------------------ init
@@ -99,6 +134,9 @@ __global__ void k_init_servers(DevParams P, StatePtrs st) {
 template <int N>
 __global__ void k_identify(DevParams P, StatePtrs st, const double *F_user, const double *p_user, int rows,
                            double *A_out, double *C_out, double *r2_out) {
+  __shared__ GridEntry sgrid[kMaxN * kMaxL];
+  load_grid(P, sgrid);
+  __syncthreads();
   const int lane = threadIdx.x & 31;
   const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (i >= P.n_srv) return;
@@ -108,7 +146,7 @@ __global__ void k_identify(DevParams P, StatePtrs st, const double *F_user, cons
   double c = 0.0;
   int nl[N];
   uint64_t key = 0;
-  double scale = P.noise_scale;
+  const double scale = P.noise_scale;
   if (synth) {
 #pragma unroll
     for (int j = 0; j < N; ++j) a[j] = st.a_true[j * ld + i];
@@ -123,7 +161,7 @@ __global__ void k_identify(DevParams P, StatePtrs st, const double *F_user, cons
       int l = -1;
       const int jv = gen_sweep_row(nl, N, r, &l);
 #pragma unroll
-      for (int j = 0; j < N; ++j) f[j] = level_value(P.k[j], j == jv ? l : P.k[j].sweep_base);
+      for (int j = 0; j < N; ++j) f[j] = sgrid[P.k[j].cls * kMaxL + (j == jv ? l : P.k[j].sweep_base)].level;
       double pw = c;
 #pragma unroll
       for (int j = 0; j < N; ++j) pw = fma(a[j], f[j], pw);
@@ -205,27 +243,11 @@ __global__ void k_identify(DevParams P, StatePtrs st, const double *F_user, cons
   }
 }
 
-__device__ __forceinline__ double demand_of(const DevParams &P, uint64_t kjit, int j, int64_t k, int burst,
-                                            double thr_max, double base, double amp) {
-  return P.demand_kind == 0 ? gen_demand_const(thr_max, P.demand_frac)
-                            : gen_demand_flag(kjit, j, k, burst, thr_max, base, amp);
-}
-
-template <int N>
-__device__ __forceinline__ uint32_t burst_mask(const DevParams &P, uint64_t kburst, int64_t epoch) {
-  uint32_t m = 0u;
-  if (P.demand_kind != 0) {
-#pragma unroll
-    for (int j = 0; j < N; ++j) m |= (uint32_t)gen_burst_flag(kburst, j, epoch) << j;
-  }
-  return m;
-}
-
 // Per instance: base cap and the virtual period -1 (Q23): u0 = f_min, acc = 0.
 template <int N>
 __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
-  __shared__ double sg[N * kMaxL];
-  for (int t = threadIdx.x; t < N * kMaxL; t += blockDim.x) sg[t] = P.g[t / kMaxL][t % kMaxL];
+  __shared__ GridEntry sgrid[kMaxN * kMaxL];
+  load_grid(P, sgrid);
   __syncthreads();
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= P.n_inst) return;
@@ -233,21 +255,25 @@ __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
   const int cidx = (int)(i % P.n_caps);
   const uint64_t srv = (uint64_t)(P.srv_begin + si);
   const int64_t ls = P.n_srv, li = P.n_inst;
-  double thr_max[N], dem[N], u0[N], acc[N], fbar[N], thr[N], a[N];
+  double thr_max[N], base[N], amp[N], dem[N], u0[N], acc[N], fbar[N], thr[N];
   const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
   const uint64_t kburst = gen_stream_key(P.seed, GEN_TAG_BURST, srv);
   const uint32_t bm = burst_mask<N>(P, kburst, 0);
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     thr_max[j] = st.thr_max[j * ls + si];
-    a[j] = st.a_true[j * ls + si];
-    dem[j] = demand_of(P, kjit, j, 0, (bm >> j) & 1u, thr_max[j], st.base[j * ls + si], st.amp[j * ls + si]);
+    base[j] = st.base[j * ls + si];
+    amp[j] = st.amp[j * ls + si];
     u0[j] = P.k[j].f_min;
     acc[j] = 0.0;
   }
-  plant_delta_sigma<N>(P, sg, u0, acc, dem, thr_max, fbar, thr, nullptr, 0);
+  demand_all<N>(P, kjit, 0, bm, thr_max, RegArr<N>{base}, RegArr<N>{amp}, dem);
+  plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
   const double noise = gen_noise(gen_stream_key(P.seed, GEN_TAG_NOISE, srv), 0, P.noise_scale);
-  st.p[i] = plant_power(st.c_true[si], a, fbar, N, noise);
+  double pw = st.c_true[si];
+#pragma unroll
+  for (int j = 0; j < N; ++j) pw = fma(st.a_true[j * ls + si], fbar[j], pw);
+  st.p[i] = pw + noise;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     st.fbar[j * li + i] = fbar[j];
@@ -260,30 +286,64 @@ __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
   for (int t = 0; t < Tri<N>::size; ++t) st.S[t * li + i] = 0.0;
   st.w[i] = 0.0;
   st.mu_p[i] = 0.0;
-  for (int t = 0; t < M; ++t) st.act[t * li + i] = 0u;
+  for (int t = 0; t < M; ++t) st.s_prev[t * li + i] = 0.0;
   const double fr = gen_cap_frac(P.seed, srv, cidx, P.cap_frac0, P.cap_frac_rand, P.cap_frac_step);
   st.cap_base[i] = gen_cap_base(st.pmin[si], st.pmax[si], fr);
 }
 
 // ------------------------------------------------------------------ shared step
 
-// One control instant for one instance: S1, S2, S3.  Returns u0 and fills
-// the trace of u/active/ahat/theta; status bits in *status.
-template <int N, int M, class SAcc, class A0Acc>
-__device__ __forceinline__ void control_instant(const DevParams &P, double cap, double &w, double (&mu_f)[N],
-                                                double &mu_p, SAcc S, double (&Sfp)[N], A0Acc A0,
-                                                const double (&fbar)[N], double p, const double (&thr)[N],
-                                                const double (&thr_max)[N], uint32_t (&act)[M],
-                                                double (&u0)[N], double (&ahat)[N], double (&theta)[N],
-                                                uint32_t &status, double *tr_u, int64_t tr_ld) {
+// Optional per-instant outputs (trace rows / control_step outputs), stride ld.
+struct InstantOut {
+  double *u, *ahat, *theta;  // [M][N], [N], [N]
+  int8_t *rank;              // [N]
+  int64_t ld;
+};
+
+// One control instant for one instance: S1, S2, S3.  Leaves u0 (block 0), the
+// roots s_t (warm starts for the next period), the per-block active codes and
+// the status; returns mean_j theta_j.  Only short-lived temporaries are kept
+// in registers (the caller's state lives in the slab / registers it owns).
+template <int N, int M, class SAcc, class VAcc, class A0Acc, class TAcc, class TmAcc>
+__device__ __forceinline__ double control_instant(const DevParams &P, double cap, double &w, VAcc mu_f,
+                                                  double &mu_p, SAcc S, VAcc Sfp, A0Acc A0,
+                                                  const double (&fbar)[N], double p, TAcc thr, TmAcc thr_max,
+                                                  double (&s_prev)[M], uint32_t (&act)[M], double (&u0)[N],
+                                                  uint32_t &status, const InstantOut &out) {
   // S1 (Eq. 5; Q1-Q4)
+  double ahat[N];
   model_push<N>(P.lam, w, mu_f, mu_p, S, Sfp, fbar, p);
   model_solve<N>(P.rho, P.a_lo, P.a_hi, S, Sfp, A0, ahat);
-  // S2
-  weights<N>(P.theta_min, thr, thr_max, theta);
-  double tau[N];
+  // S2: theta (IEEE division), tau_j = ahat_j / R_j = ahat_j theta_j / r0_j
+  double tau[N], tsum = 0.0;
+  {
+    double th[N], tr_[N], tm_[N];
 #pragma unroll
-  for (int j = 0; j < N; ++j) tau[j] = ahat[j] * theta[j] * P.k[j].inv_r0;
+    for (int j = 0; j < N; ++j) {
+      tr_[j] = thr.get(j);
+      tm_[j] = thr_max.get(j);
+    }
+    weights<N>(P.theta_min, tr_, tm_, th);
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      tsum += th[j];
+      tau[j] = ahat[j] * th[j] * P.k[j].inv_r0;
+    }
+    if (out.theta) {
+#pragma unroll
+      for (int j = 0; j < N; ++j) out.theta[j * out.ld] = th[j];
+    }
+    if (out.rank) {
+      int8_t rk[N];
+      ranks<N>(th, rk);
+#pragma unroll
+      for (int j = 0; j < N; ++j) out.rank[j * out.ld] = rk[j];
+    }
+  }
+  if (out.ahat) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) out.ahat[j * out.ld] = ahat[j];
+  }
   // S3 (Eq. 9-10a)
   double beta = p - cap, smin = 0.0, smax = 0.0;
 #pragma unroll
@@ -292,65 +352,85 @@ __device__ __forceinline__ void control_instant(const DevParams &P, double cap, 
     smin = fma(ahat[j], P.k[j].lo, smin);
     smax = fma(ahat[j], P.k[j].hi, smax);
   }
-  status = 0u;
-  if (beta + smin > 0.0 || beta + smax < 0.0) status |= CAPGPU_ST_CAP_INFEASIBLE;
-  bool capped = false;
-#pragma unroll
+  status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
+  // Blocks t = 0..M-1, one loop body (not unrolled: instruction cache); the
+  // per-block registers rotate so the body indexes no array by t.
+#pragma unroll 1
   for (int t = 0; t < M; ++t) {
+    double ctau[N];
+    const double c = P.ct[t];
+#pragma unroll
+    for (int j = 0; j < N; ++j) ctau[j] = c * tau[j];
+    const double s = P.convex ? solve_block_convex<N>(P.k, ahat, ctau, beta, smin, s_prev[0])
+                              : solve_block<N>(P.k, P.k_dev, ahat, ctau, beta, s_prev[0]);
     double u[N];
-    act[t] = solve_block<N>(P.k, ahat, tau, P.ct[t], beta, act[t], u, capped);
+    const uint32_t code = block_u<N>(P.k, ctau, s, u);
     if (t == 0) {
 #pragma unroll
       for (int j = 0; j < N; ++j) u0[j] = u[j];
     }
-    if (tr_u) {
+    if (out.u) {
 #pragma unroll
-      for (int j = 0; j < N; ++j) tr_u[(int64_t)(t * N + j) * tr_ld] = u[j];
+      for (int j = 0; j < N; ++j) out.u[(int64_t)(t * N + j) * out.ld] = u[j];
     }
+#pragma unroll
+    for (int q = 0; q + 1 < M; ++q) {
+      s_prev[q] = s_prev[q + 1];
+      act[q] = act[q + 1];
+    }
+    s_prev[M - 1] = s;
+    act[M - 1] = code;
   }
-  if (capped) status |= CAPGPU_ST_SOLVER_CAP;
+  return tsum * P.inv_N;
 }
 
 // ------------------------------------------------------------------ fused simulate
 
-// Slab fields (per thread): S[T] | A0[N] | a_true[N] | thr_max[N] | base[N] | amp[N]
+// Slab fields (per thread, AoS):
+//   S[T] | mu_f[N] | Sfp[N] | A0[N] | a_true[N] | thr_max[N] | base[N] | amp[N]
+// (the model scatter and the read-only constants; fbar, acc, thr stay in
+// registers next to the LDL^T working set).
 template <int N>
-struct Slab {
+struct SlabLayout {
   static constexpr int T = Tri<N>::size;
-  static constexpr int fields = T + 5 * N;
+  static constexpr int used = T + 7 * N;
+  static constexpr int F = used | 1;  // odd stride: conflict-free 8-byte accesses
+  static constexpr int oMU = T, oSFP = T + N, oA0 = T + 2 * N, oAT = T + 3 * N, oTM = T + 4 * N,
+                       oBA = T + 5 * N, oAM = T + 6 * N;
 };
 
-template <int N, int M>
-__global__ void __launch_bounds__(128) k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
-  extern __shared__ double slab_mem[];
-  __shared__ double sg[N * kMaxL];
-  for (int t = threadIdx.x; t < N * kMaxL; t += blockDim.x) sg[t] = P.g[t / kMaxL][t % kMaxL];
+template <int N, int M, int S, int BLOCK>
+__global__ void __launch_bounds__(BLOCK) k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
+  using SL = SlabLayout<N>;
+  extern __shared__ __align__(16) double smem[];
+  GridEntry *sgrid = reinterpret_cast<GridEntry *>(smem);
+  load_grid(P, sgrid);
   __syncthreads();
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x;
   if (i >= P.n_inst) return;
-  constexpr int T = Slab<N>::T;
-  const int stride = blockDim.x;
-  double *my = slab_mem + threadIdx.x;
-  const SlabAcc S{my, stride};
-  const SlabAcc A0{my + T * stride, stride};
-  const SlabAcc AT{my + (T + N) * stride, stride};
-  const SlabAcc TM{my + (T + 2 * N) * stride, stride};
-  const SlabAcc BA{my + (T + 3 * N) * stride, stride};
-  const SlabAcc AM{my + (T + 4 * N) * stride, stride};
+  double *my = smem + 4 * P.n_class * kMaxL + threadIdx.x * SL::F;
+  const Slab Sm{my};
+  const Slab MU{my + SL::oMU};
+  const Slab SF{my + SL::oSFP};
+  const Slab A0{my + SL::oA0};
+  const Slab AT{my + SL::oAT};
+  const Slab TM{my + SL::oTM};
+  const Slab BA{my + SL::oBA};
+  const Slab AM{my + SL::oAM};
 
-  const int64_t si = i / P.n_caps;
+  int64_t si = i / P.n_caps;
   const uint64_t srv = (uint64_t)(P.srv_begin + si);
-  const int64_t ls = P.n_srv, li = P.n_inst;
+  int64_t ls = P.n_srv, li = P.n_inst;
 
   // ---- stage state into registers / slab
-  double fbar[N], acc[N], thr[N], mu_f[N], Sfp[N];
+  double fbar[N], acc[N], thr[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     fbar[j] = st.fbar[j * li + i];
     acc[j] = st.acc[j * li + i];
     thr[j] = st.thr[j * li + i];
-    mu_f[j] = st.mu_f[j * li + i];
-    Sfp[j] = st.Sfp[j * li + i];
+    MU.set(j, st.mu_f[j * li + i]);
+    SF.set(j, st.Sfp[j * li + i]);
     A0.set(j, st.A0[j * ls + si]);
     AT.set(j, st.a_true[j * ls + si]);
     TM.set(j, st.thr_max[j * ls + si]);
@@ -358,38 +438,45 @@ __global__ void __launch_bounds__(128) k_simulate(DevParams P, StatePtrs st, Tra
     AM.set(j, st.amp[j * ls + si]);
   }
 #pragma unroll
-  for (int t = 0; t < T; ++t) S.set(t, st.S[t * li + i]);
+  for (int t = 0; t < SL::T; ++t) Sm.set(t, st.S[t * li + i]);
   double p = st.p[i], w = st.w[i], mu_p = st.mu_p[i];
   const double c_true = st.c_true[si], cap_base = st.cap_base[i];
-  uint32_t act[M];
+  double s_prev[M];
 #pragma unroll
-  for (int t = 0; t < M; ++t) act[t] = st.act[t * li + i];
+  for (int t = 0; t < M; ++t) s_prev[t] = st.s_prev[t * li + i];
   const int slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
   const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
   const uint64_t kburst = gen_stream_key(P.seed, GEN_TAG_BURST, srv);
   const uint64_t knoise = gen_stream_key(P.seed, GEN_TAG_NOISE, srv);
-  int64_t epoch = -1;
-  uint32_t bmask = 0u;
+  // burst epoch of period k0 + 1 and periods left in it
+  int64_t epoch = (k0 + 1) / GEN_BURST_HOLD;
+  int left = (int)(GEN_BURST_HOLD - (k0 + 1) % GEN_BURST_HOLD);
+  uint32_t bmask = burst_mask<N>(P, kburst, epoch);
 
   // ---- summaries (Q25)
   const int kw = K - (4 * K) / 5;
-  double sum_p = 0.0, sumsq_p = 0.0, max_p = -INFINITY, sum_theta = 0.0;
-  int n_viol = 0, n_win = 0;
+  double sum_p = 0.0, sumsq_p = 0.0, max_p = 0.0, sum_theta = 0.0;
+  int n_viol = 0;
   int act_cnt[M];
 #pragma unroll
   for (int t = 0; t < M; ++t) act_cnt[t] = 0;
 
+#pragma unroll 1
   for (int kk = 0; kk < K; ++kk) {
     const int64_t k = k0 + kk;
     const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
-    double thr_max[N];
-#pragma unroll
-    for (int j = 0; j < N; ++j) thr_max[j] = TM.get(j);
-    double u0[N], ahat[N], theta[N];
-    uint32_t status;
-    double *tr_u = slot >= 0 && tr.u ? tr.u + (int64_t)kk * M * N * tr.n_trace + slot : nullptr;
-    control_instant<N, M>(P, cap, w, mu_f, mu_p, S, Sfp, A0, fbar, p, thr, thr_max, act, u0, ahat, theta,
-                          status, tr_u, tr.n_trace);
+    double u0[N];
+    uint32_t status, act[M];
+    InstantOut io{};
+    if (slot >= 0) {
+      io.ld = tr.n_trace;
+      io.u = tr.u ? tr.u + (int64_t)kk * M * N * tr.n_trace + slot : nullptr;
+      io.ahat = tr.ahat ? tr.ahat + (int64_t)kk * N * tr.n_trace + slot : nullptr;
+      io.theta = tr.theta ? tr.theta + (int64_t)kk * N * tr.n_trace + slot : nullptr;
+      io.rank = tr.rank ? tr.rank + (int64_t)kk * N * tr.n_trace + slot : nullptr;
+    }
+    const double tbar = control_instant<N, M>(P, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
+                                              act, u0, status, io);
     if (slot >= 0) {
       const int64_t b = (int64_t)kk * tr.n_trace + slot;
       if (tr.p) tr.p[b] = p;
@@ -399,69 +486,70 @@ __global__ void __launch_bounds__(128) k_simulate(DevParams P, StatePtrs st, Tra
 #pragma unroll
         for (int t = 0; t < M; ++t) tr.active[((int64_t)kk * M + t) * tr.n_trace + slot] = act[t];
       }
-      int8_t rk[N];
-      ranks<N>(theta, rk);
-#pragma unroll
-      for (int j = 0; j < N; ++j) {
-        const int64_t e = ((int64_t)kk * N + j) * tr.n_trace + slot;
-        if (tr.ahat) tr.ahat[e] = ahat[j];
-        if (tr.theta) tr.theta[e] = theta[j];
-        if (tr.rank) tr.rank[e] = rk[j];
-      }
     }
-    // ---- S4: period k -> k+1
-    const int64_t kn = k + 1;
-    if (kn / GEN_BURST_HOLD != epoch) {
-      epoch = kn / GEN_BURST_HOLD;
+    // ---- S4: period k -> k+1 (demand and meter noise of period k+1)
+    if (left == 0) {
+      ++epoch;
+      left = GEN_BURST_HOLD;
       bmask = burst_mask<N>(P, kburst, epoch);
     }
-    double dem[N];
+    --left;
+    double dem[N], thr_max[N];
 #pragma unroll
-    for (int j = 0; j < N; ++j) dem[j] = demand_of(P, kjit, j, kn, (bmask >> j) & 1u, thr_max[j], BA.get(j), AM.get(j));
-    uint8_t *lv = slot >= 0 && tr.levels ? tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot : nullptr;
-    plant_delta_sigma<N>(P, sg, u0, acc, dem, thr_max, fbar, thr, lv, tr.n_trace);
-    const double noise = gen_noise(knoise, kn, P.noise_scale);
+    for (int j = 0; j < N; ++j) thr_max[j] = TM.get(j);
+    demand_all<N>(P, kjit, k + 1, bmask, thr_max, BA, AM, dem);
+    if (slot >= 0 && tr.levels) {
+      double u_l[N], a_l[N];
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        u_l[j] = u0[j];
+        a_l[j] = acc[j];
+      }
+      plant_trace_levels<N>(P.k_dev, P.S, sgrid, u_l, a_l, tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot,
+                            tr.n_trace);
+    }
+    plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+    const double noise = gen_noise(knoise, k + 1, P.noise_scale);
     double pw = c_true;
 #pragma unroll
     for (int j = 0; j < N; ++j) pw = fma(AT.get(j), fbar[j], pw);
     p = pw + noise;
     if (kk >= kw) {
-      double tb = 0.0;
-#pragma unroll
-      for (int j = 0; j < N; ++j) tb += theta[j];
-      sum_theta += tb / (double)N;
+      sum_theta += tbar;
       sum_p += p;
       sumsq_p = fma(p, p, sumsq_p);
-      max_p = fmax(max_p, p);
+      max_p = kk == kw ? p : fmax(max_p, p);
       n_viol += p > cap;
-      ++n_win;
 #pragma unroll
       for (int t = 0; t < M; ++t) act_cnt[t] += act[t] != 0u;
     }
   }
 
-  // ---- write back
+  // ---- write back.  Launder the indices so the compiler recomputes the ~100
+  // state addresses here instead of keeping the stage-in ones alive (spilled)
+  // across the whole period loop.
+  asm volatile("" : "+l"(i), "+l"(li), "+l"(ls), "+l"(si));
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     st.fbar[j * li + i] = fbar[j];
     st.acc[j * li + i] = acc[j];
     st.thr[j * li + i] = thr[j];
-    st.mu_f[j * li + i] = mu_f[j];
-    st.Sfp[j * li + i] = Sfp[j];
+    st.mu_f[j * li + i] = MU.get(j);
+    st.Sfp[j * li + i] = SF.get(j);
   }
 #pragma unroll
-  for (int t = 0; t < T; ++t) st.S[t * li + i] = S.get(t);
+  for (int t = 0; t < SL::T; ++t) st.S[t * li + i] = Sm.get(t);
   st.p[i] = p;
   st.w[i] = w;
   st.mu_p[i] = mu_p;
 #pragma unroll
-  for (int t = 0; t < M; ++t) st.act[t * li + i] = act[t];
+  for (int t = 0; t < M; ++t) st.s_prev[t * li + i] = s_prev[t];
   if (tr.sum_p) tr.sum_p[i] = sum_p;
   if (tr.sumsq_p) tr.sumsq_p[i] = sumsq_p;
   if (tr.max_p) tr.max_p[i] = max_p;
   if (tr.sum_theta) tr.sum_theta[i] = sum_theta;
   if (tr.n_viol) tr.n_viol[i] = n_viol;
-  if (tr.n_window) tr.n_window[i] = n_win;
+  if (tr.n_window) tr.n_window[i] = K - kw;
   if (tr.final_p) tr.final_p[i] = p;
   if (tr.act_count) {
 #pragma unroll
@@ -489,23 +577,20 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
     fbar[j] = f_app[j * ld + i];
     thr[j] = thr_in[j * ld + i];
     thr_max[j] = thr_max_in[j * ld + i];
-    finite &= isfinite(fbar[j]) && isfinite(thr[j]) && isfinite(thr_max[j]) && thr_max[j] > 0.0;
+    finite &= isfinite(fbar[j]) && isfinite(thr[j]) && isfinite(thr_max[j]) && thr_max[j] > 0.0 && thr[j] >= 0.0;
     mu_f[j] = st.mu_f[j * ld + i];
     Sfp[j] = st.Sfp[j * ld + i];
     A0r[j] = st.A0[j * ld + i];
   }
-  uint32_t act[M];
-#pragma unroll
-  for (int t = 0; t < M; ++t) act[t] = st.act[t * ld + i];
   if (!finite) {
     // Q26: hold the model, pin outputs to the lower bounds
+    uint32_t all = 0u;
+#pragma unroll
+    for (int j = 0; j < N; ++j) all |= 1u << (2 * j);
 #pragma unroll
     for (int t = 0; t < M; ++t) {
 #pragma unroll
       for (int j = 0; j < N; ++j) u_out[((int64_t)t * N + j) * ld + i] = P.k[j].lo;
-      uint32_t all = 0u;
-#pragma unroll
-      for (int j = 0; j < N; ++j) all |= 1u << (2 * j);
       act_out[(int64_t)t * ld + i] = all;
     }
     if (status_out) status_out[i] = CAPGPU_ST_NONFINITE;
@@ -520,11 +605,15 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
     return;
   }
   double w = st.w[i], mu_p = st.mu_p[i];
+  double s_prev[M];
+#pragma unroll
+  for (int t = 0; t < M; ++t) s_prev[t] = st.s_prev[t * ld + i];
   const GlobAcc S{st.S + i, ld};
-  double u0[N], ahat[N], theta[N];
-  uint32_t status;
-  control_instant<N, M>(P, cap, w, mu_f, mu_p, S, Sfp, RegArr<N>{A0r}, fbar, p, thr, thr_max, act, u0, ahat,
-                        theta, status, u_out + i, ld);
+  double u0[N];
+  uint32_t status, act[M];
+  InstantOut io{u_out + i, ahat_out ? ahat_out + i : nullptr, nullptr, rank_out ? rank_out + i : nullptr, ld};
+  control_instant<N, M>(P, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
+                        RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
   st.w[i] = w;
   st.mu_p[i] = mu_p;
 #pragma unroll
@@ -534,20 +623,10 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
   }
 #pragma unroll
   for (int t = 0; t < M; ++t) {
-    st.act[t * ld + i] = act[t];
+    st.s_prev[t * ld + i] = s_prev[t];
     act_out[(int64_t)t * ld + i] = act[t];
   }
   if (status_out) status_out[i] = status;
-  if (ahat_out) {
-#pragma unroll
-    for (int j = 0; j < N; ++j) ahat_out[j * ld + i] = ahat[j];
-  }
-  if (rank_out) {
-    int8_t rk[N];
-    ranks<N>(theta, rk);
-#pragma unroll
-    for (int j = 0; j < N; ++j) rank_out[j * ld + i] = rk[j];
-  }
 }
 
 template <int N>
@@ -585,14 +664,18 @@ __global__ void k_debug_gen(DevParams P, StatePtrs st, int64_t k, double *a_true
   const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
   const uint64_t kburst = gen_stream_key(P.seed, GEN_TAG_BURST, srv);
   const uint32_t bm = burst_mask<N>(P, kburst, k / GEN_BURST_HOLD);
+  double tm[N], ba[N], am[N], d[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    const double tm = gen_thr_max(P.seed, srv, j);
+    tm[j] = gen_thr_max(P.seed, srv, j);
+    ba[j] = gen_dem_base(P.seed, srv, j);
+    am[j] = gen_dem_amp(P.seed, srv, j);
     a_true[j * ld + i] = gen_a_true(P.seed, srv, j);
-    thr_max[j * ld + i] = tm;
-    dem[j * ld + i] = demand_of(P, kjit, j, k, (bm >> j) & 1u, tm, gen_dem_base(P.seed, srv, j),
-                                gen_dem_amp(P.seed, srv, j));
+    thr_max[j * ld + i] = tm[j];
   }
+  demand_all<N>(P, kjit, k, bm, tm, RegArr<N>{ba}, RegArr<N>{am}, d);
+#pragma unroll
+  for (int j = 0; j < N; ++j) dem[j * ld + i] = d[j];
   c_true[i] = gen_c_true(P.seed, srv);
   noise[i] = gen_noise(gen_stream_key(P.seed, GEN_TAG_NOISE, srv), k, P.noise_scale);
 }
@@ -612,7 +695,6 @@ struct Launchers {
                         cudaStream_t);
   int (*debug_gen)(const DevParams &, const StatePtrs &, int64_t, double *, double *, double *, double *, double *,
                    cudaStream_t);
-  int (*sim_smem_bytes)(int block);
 };
 
 inline int grid_for(int64_t n, int block) { return (int)((n + block - 1) / block); }
@@ -642,22 +724,62 @@ struct LaunchN {
     k_debug_gen<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, k, a, tm, c, dem, noise);
     return (int)cudaGetLastError();
   }
-  static int sim_smem_bytes(int block) { return (int)(sizeof(double) * Slab<N>::fields * block); }
 };
+
+// Fused-kernel launch: block size chosen so that the last wave is nearly full
+// (the per-instance period chain is serial, so a ragged last wave costs a
+// whole per-instance run time).
+template <int N, int M, int S, int BLOCK>
+int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
+  const int smem = (int)(sizeof(double) * (4 * P.n_class * kMaxL + SlabLayout<N>::F * BLOCK));
+  cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  k_simulate<N, M, S, BLOCK><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
+  return (int)cudaGetLastError();
+}
+
+template <int N, int M, int S>
+int sim_occupancy(int block, int n_class) {
+  int nb = 0;
+  const int smem_per_block = (int)(sizeof(double) * (4 * n_class * kMaxL + SlabLayout<N>::F * block));
+  if (block == 32) {
+    cudaFuncSetAttribute(k_simulate<N, M, S, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 32>, 32, smem_per_block);
+  } else {
+    cudaFuncSetAttribute(k_simulate<N, M, S, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 128>, 128, smem_per_block);
+  }
+  return nb;
+}
 
 template <int N, int M>
 struct LaunchNM {
+  template <int S>
+  static int sim_s(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
+    // waves = n_inst / (SMs * threads resident per SM); pick the block size
+    // whose last wave is fuller (ties -> 128).
+    static int sms = 0, occ32[kMaxN + 1] = {0}, occ128[kMaxN + 1] = {0};
+    const int nc = P.n_class;
+    if (!sms) {
+      int dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    if (!occ128[nc]) {
+      occ32[nc] = sim_occupancy<N, M, S>(32, nc);
+      occ128[nc] = sim_occupancy<N, M, S>(128, nc);
+    }
+    // a per-instance run is a serial chain: time ~ number of waves
+    auto waves = [&](int occ, int block) {
+      const double slots = (double)sms * occ * block;
+      return slots <= 0 ? 1e30 : std::ceil((double)P.n_inst / slots);
+    };
+    if (occ128[nc] <= 0 || waves(occ32[nc], 32) < waves(occ128[nc], 128))
+      return launch_sim<N, M, S, 32>(P, st, tr, k0, K, s);
+    return launch_sim<N, M, S, 128>(P, st, tr, k0, K, s);
+  }
   static int simulate(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K,
                       cudaStream_t s) {
-    const int block = 128;
-    const int smem = LaunchN<N>::sim_smem_bytes(block);
-    static bool attr = false;
-    if (!attr) {
-      cudaFuncSetAttribute(k_simulate<N, M>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-      attr = true;
-    }
-    k_simulate<N, M><<<grid_for(P.n_inst, block), block, smem, s>>>(P, st, tr, k0, K);
-    return (int)cudaGetLastError();
+    return sim_s<0>(P, st, tr, k0, K, s);
   }
   static int control_step(const DevParams &P, const StatePtrs &st, const double *p, const double *f,
                           const double *thr, const double *tm, const double *cap, double *u, uint32_t *act,
@@ -676,7 +798,6 @@ Launchers make_launchers(int M) {
   L.init_instances = &LaunchN<N>::init_instances;
   L.assign_weights = &LaunchN<N>::assign_weights;
   L.debug_gen = &LaunchN<N>::debug_gen;
-  L.sim_smem_bytes = &LaunchN<N>::sim_smem_bytes;
   switch (M) {
     case 1: L.simulate = &LaunchNM<N, 1>::simulate; L.control_step = &LaunchNM<N, 1>::control_step; break;
     case 2: L.simulate = &LaunchNM<N, 2>::simulate; L.control_step = &LaunchNM<N, 2>::control_step; break;

@@ -250,6 +250,18 @@ def test_closed_loop_shapes(G, oracle_mod, n_gpus, P, M, n):
     _sim_compare(G, oracle_mod, d, n, np.array([0, n // 2, n - 1]), periods=150)
 
 
+@pytest.mark.parametrize("n_gpus,M", [(2, 2), (8, 3)])
+def test_closed_loop_slo_lower_bounds(G, oracle_mod, n_gpus, M):
+    """SLO-raised lower bounds l_j > f_min (Eq. 10b-c, Q14) make the block QP
+    non-convex in s: exercises the general (safeguarded + exact breakpoint) solve."""
+    d = desc_for(n_gpus, P=8, M=M, periods=200)
+    for j, k in enumerate(d["knobs"]):
+        if j >= 1:
+            k["f_lo"] = 600.0 + 40.0 * j  # GPU j must run >= 640.. MHz to meet its SLO
+    d["workload"].update(demand_kind=1, cap_frac0=0.1, cap_frac_rand=0.8)
+    _sim_compare(G, oracle_mod, d, 97, np.array([0, 13, 96]), periods=200)
+
+
 def test_closed_loop_infeasible_caps(G, oracle_mod):
     """Caps below P_min / above P_max: CAP_INFEASIBLE and the frequencies pin to
     the box."""
