@@ -270,6 +270,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     k.lo = b.f_lo == 0.0 ? b.f_min : b.f_lo;
     k.hi = b.f_max;
     k.m = b.f_min;  // Q7
+    k.span = k.hi - k.m;
     k.r0 = b.r0 == 0.0 ? prm.r0 : b.r0;
     k.inv_r0 = 1.0 / k.r0;
   }
@@ -281,7 +282,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   const int64_t nd_inst = (int64_t)(5 * N + c->T + 4);
   const int64_t nd_srv = (int64_t)(5 * N + 3);
   const int64_t grid_bytes = (int64_t)sizeof(GridEntry) * n_class * CAPGPU_MAX_LEVELS;
-  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 8 * (int64_t)h.M * ni + 4 * ni + grid_bytes +
+  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 12 * (int64_t)h.M * ni + 4 * ni + grid_bytes +
                         (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 256;
   cudaError_t e = cudaMalloc(&c->ws, (size_t)bytes);
   if (e != cudaSuccess) {
@@ -318,6 +319,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice);
   d.k_dev = kdev;
   s.trace_slot = (int32_t *)q;
+  s.act = (uint32_t *)(s.trace_slot + ni);
   for (int c2 = 0; c2 < n_class; ++c2)
     cudaMemcpy(gdev + c2 * CAPGPU_MAX_LEVELS, grid[c2], sizeof(GridEntry) * CAPGPU_MAX_LEVELS,
                cudaMemcpyHostToDevice);
@@ -398,6 +400,7 @@ int capgpu_model_reset(capgpu_ctx *c, void *stream) {
   CK_CUDA(c, cudaMemsetAsync(c->st.S, 0, sizeof(double) * c->T * ni, s));
   CK_CUDA(c, cudaMemsetAsync(c->st.Sfp, 0, sizeof(double) * c->N * ni, s));
   CK_CUDA(c, cudaMemsetAsync(c->st.s_prev, 0, sizeof(double) * c->M * ni, s));
+  CK_CUDA(c, cudaMemsetAsync(c->st.act, 0, sizeof(uint32_t) * c->M * ni, s));
   return CAPGPU_OK;
 }
 

@@ -43,6 +43,7 @@ struct Tri {
 struct KnobConst {
   double f_min, f_max, step, inv_step;  // grid (Q15)
   double lo, hi, m;                     // box [l, h] (Eq. 10a, Q14) and penalty reference f_min (Q7)
+  double span;                          // hi - m
   double r0, inv_r0;                    // r0_j and 1 / r0_j (Q6, Q9)
   int32_t L;                            // levels
   int32_t sweep_base;
@@ -314,49 +315,56 @@ __device__ __noinline__ double block_exact(const KnobConst *kc, const double *a_
 }
 
 // Convex case (no SLO-raised lower bound: lo_j == m_j for all j).  For s >= 0
-// every knob sits at lo, so phi(s) = s - beta - a.lo there; for s < 0 each
-// u_j(s) = min(m_j - c tau_j s, hi_j) and phi is convex.  Hence:
-//   phi(0) <= 0  ->  s* = beta + a.lo >= 0 exactly (all knobs at lo);
-//   otherwise Newton from the right of the root converges monotonically (a
-//   start left of the root overshoots once to the right), each step landing
-//   on the root of the current piece; it ends when the new point stays in
-//   the piece (exact).  At most N + 2 steps, no safeguard needed.
-// a_lo_sum = sum_j a_j lo_j (shared by the blocks of an instant).
+// every knob sits at lo (phi(s) = s - beta - a.lo); for s < 0 every knob is
+// free or at its upper bound, u_j(s) = min(m_j - c tau_j s, hi_j), and phi is
+// convex.  Hence:
+//   beta + a.lo >= 0  ->  s* = beta + a.lo exactly (all knobs at lo);
+//   otherwise the piece with upper set U has the root
+//     s_U = (beta + a.lo + sum_{j in U} a_j (hi_j - m_j)) / (1 + sum_{j not in U} c tau_j a_j)
+//   and, phi being convex, every piece line lies below phi, so s_U >= s*.
+//   Starting from last period's U, s_U >= s* and U(s_U) is a subset of U(s*);
+//   iterating U <- U(s_U) moves s down monotonically and stops exactly when
+//   the set reproduces itself: the exact root, in at most N + 1 steps.
+// No phi evaluation is needed: one piece root and one classification per step.
+// code: in = previous period's codes of this block, out = codes at the root.
 template <int N>
 __device__ __forceinline__ double solve_block_convex(const KnobConst *kc, const double (&a)[N],
-                                                     const double (&ctau)[N], double beta, double a_lo_sum,
-                                                     double s_warm) {
-  const double phi0 = -(beta + a_lo_sum);
-  if (!(phi0 > 0.0)) return beta + a_lo_sum;
-  double cta[N], sum_cta = 1.0;
+                                                     const double (&ad)[N], const double (&ctau)[N],
+                                                     double beta, double a_lo_sum, uint32_t &code) {
+  const double base = beta + a_lo_sum;
+  if (!(base < 0.0)) {
+    uint32_t c = 0u;
+#pragma unroll
+    for (int j = 0; j < N; ++j) c |= (base > 0.0 && ctau[j] > 0.0 ? 1u : 0u) << (2 * j);
+    code = c;
+    return base;
+  }
+  double cta[N], den_all = 1.0;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     cta[j] = ctau[j] * a[j];
-    sum_cta += cta[j];
+    den_all += cta[j];
   }
-  double s, phi, slope;
-  uint32_t code;
-  if (s_warm < 0.0) {
-    s = s_warm;
-    code = block_eval<N>(kc, a, ctau, cta, beta, s, phi, slope);
-  } else {  // just left of 0: every knob free
-    s = 0.0;
-    phi = phi0;
-    slope = sum_cta;
-    code = 0u;
-  }
+  uint32_t up = code & 0xAAAAAAAAu;  // previous upper set (bit 2j+1)
+  double s = 0.0;
 #pragma unroll 1
-  for (int it = 0; it < N + 2; ++it) {
-    if (phi == 0.0) return s;
-    double s1 = fma(-phi, rcp_fast(slope), s);
-    if (s1 >= 0.0) {  // overshoot from the left: restart just left of 0
-      s1 = -phi0 * rcp_fast(sum_cta);
-      code = 0u;
+  for (int it = 0; it <= N; ++it) {
+    double num = base, den = den_all;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      if ((up >> (2 * j + 1)) & 1u) {
+        num += ad[j];
+        den -= cta[j];
+      }
     }
-    if (block_codes<N>(kc, ctau, s1) == code) return s1;
-    s = s1;
-    code = block_eval<N>(kc, a, ctau, cta, beta, s, phi, slope);
+    s = num * rcp_fast(den);
+    uint32_t nu = 0u;
+#pragma unroll
+    for (int j = 0; j < N; ++j) nu |= (fma(-ctau[j], s, kc[j].m) > kc[j].hi ? 2u : 0u) << (2 * j);
+    if (nu == up) break;
+    up = nu;
   }
+  code = up;
   return s;
 }
 

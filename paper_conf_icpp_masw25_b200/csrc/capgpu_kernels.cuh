@@ -26,6 +26,7 @@ struct StatePtrs {
   double *fbar, *acc, *thr, *p;            // plant state S4
   double *w, *mu_f, *mu_p, *S, *Sfp;       // model state S1
   double *s_prev;                          // [M] warm-start roots of the block QPs
+  uint32_t *act;                           // [M] warm-start active codes of the block QPs
   double *cap_base;                        // [1]
   int32_t *trace_slot;                     // [1] -1 = not traced
   // per server (ld = n_srv)
@@ -286,7 +287,10 @@ __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
   for (int t = 0; t < Tri<N>::size; ++t) st.S[t * li + i] = 0.0;
   st.w[i] = 0.0;
   st.mu_p[i] = 0.0;
-  for (int t = 0; t < M; ++t) st.s_prev[t * li + i] = 0.0;
+  for (int t = 0; t < M; ++t) {
+    st.s_prev[t * li + i] = 0.0;
+    st.act[t * li + i] = 0u;
+  }
   const double fr = gen_cap_frac(P.seed, srv, cidx, P.cap_frac0, P.cap_frac_rand, P.cap_frac_step);
   st.cap_base[i] = gen_cap_base(st.pmin[si], st.pmax[si], fr);
 }
@@ -354,24 +358,36 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double cap
   }
   status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
   // Blocks t = 0..M-1, one loop body (not unrolled: instruction cache); the
-  // per-block registers rotate so the body indexes no array by t.
+  // per-block registers rotate so the body indexes no array by t.  act[] holds
+  // last period's codes on entry (warm start) and this period's on exit.
+  double ad[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) ad[j] = ahat[j] * P.k[j].span;
 #pragma unroll 1
   for (int t = 0; t < M; ++t) {
     double ctau[N];
     const double c = P.ct[t];
 #pragma unroll
     for (int j = 0; j < N; ++j) ctau[j] = c * tau[j];
-    const double s = P.convex ? solve_block_convex<N>(P.k, ahat, ctau, beta, smin, s_prev[0])
-                              : solve_block<N>(P.k, P.k_dev, ahat, ctau, beta, s_prev[0]);
-    double u[N];
-    const uint32_t code = block_u<N>(P.k, ctau, s, u);
-    if (t == 0) {
-#pragma unroll
-      for (int j = 0; j < N; ++j) u0[j] = u[j];
+    uint32_t code = act[0];
+    double s;
+    if (P.convex) {
+      s = solve_block_convex<N>(P.k, ahat, ad, ctau, beta, smin, code);
+    } else {
+      s = solve_block<N>(P.k, P.k_dev, ahat, ctau, beta, s_prev[0]);
+      code = block_codes<N>(P.k, ctau, s);
     }
-    if (out.u) {
+    if (t == 0 || out.u) {
+      double u[N];
+      code = block_u<N>(P.k, ctau, s, u);
+      if (t == 0) {
 #pragma unroll
-      for (int j = 0; j < N; ++j) out.u[(int64_t)(t * N + j) * out.ld] = u[j];
+        for (int j = 0; j < N; ++j) u0[j] = u[j];
+      }
+      if (out.u) {
+#pragma unroll
+        for (int j = 0; j < N; ++j) out.u[(int64_t)(t * N + j) * out.ld] = u[j];
+      }
     }
 #pragma unroll
     for (int q = 0; q + 1 < M; ++q) {
@@ -443,7 +459,12 @@ __global__ void __launch_bounds__(BLOCK) k_simulate(DevParams P, StatePtrs st, T
   const double c_true = st.c_true[si], cap_base = st.cap_base[i];
   double s_prev[M];
 #pragma unroll
-  for (int t = 0; t < M; ++t) s_prev[t] = st.s_prev[t * li + i];
+  uint32_t act[M];
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+    s_prev[t] = st.s_prev[t * li + i];
+    act[t] = st.act[t * li + i];
+  }
   const int slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
   const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
   const uint64_t kburst = gen_stream_key(P.seed, GEN_TAG_BURST, srv);
@@ -466,7 +487,7 @@ __global__ void __launch_bounds__(BLOCK) k_simulate(DevParams P, StatePtrs st, T
     const int64_t k = k0 + kk;
     const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
     double u0[N];
-    uint32_t status, act[M];
+    uint32_t status;
     InstantOut io{};
     if (slot >= 0) {
       io.ld = tr.n_trace;
@@ -543,7 +564,10 @@ __global__ void __launch_bounds__(BLOCK) k_simulate(DevParams P, StatePtrs st, T
   st.w[i] = w;
   st.mu_p[i] = mu_p;
 #pragma unroll
-  for (int t = 0; t < M; ++t) st.s_prev[t * li + i] = s_prev[t];
+  for (int t = 0; t < M; ++t) {
+    st.s_prev[t * li + i] = s_prev[t];
+    st.act[t * li + i] = act[t];
+  }
   if (tr.sum_p) tr.sum_p[i] = sum_p;
   if (tr.sumsq_p) tr.sumsq_p[i] = sumsq_p;
   if (tr.max_p) tr.max_p[i] = max_p;
@@ -606,11 +630,14 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
   }
   double w = st.w[i], mu_p = st.mu_p[i];
   double s_prev[M];
+  uint32_t status, act[M];
 #pragma unroll
-  for (int t = 0; t < M; ++t) s_prev[t] = st.s_prev[t * ld + i];
+  for (int t = 0; t < M; ++t) {
+    s_prev[t] = st.s_prev[t * ld + i];
+    act[t] = st.act[t * ld + i];
+  }
   const GlobAcc S{st.S + i, ld};
   double u0[N];
-  uint32_t status, act[M];
   InstantOut io{u_out + i, ahat_out ? ahat_out + i : nullptr, nullptr, rank_out ? rank_out + i : nullptr, ld};
   control_instant<N, M>(P, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
                         RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
@@ -624,6 +651,7 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
 #pragma unroll
   for (int t = 0; t < M; ++t) {
     st.s_prev[t * ld + i] = s_prev[t];
+    st.act[t * ld + i] = act[t];
     act_out[(int64_t)t * ld + i] = act[t];
   }
   if (status_out) status_out[i] = status;
@@ -768,12 +796,16 @@ struct LaunchNM {
       occ32[nc] = sim_occupancy<N, M, S>(32, nc);
       occ128[nc] = sim_occupancy<N, M, S>(128, nc);
     }
-    // a per-instance run is a serial chain: time ~ number of waves
-    auto waves = [&](int occ, int block) {
-      const double slots = (double)sms * occ * block;
-      return slots <= 0 ? 1e30 : std::ceil((double)P.n_inst / slots);
+    // The SM throughput is shared by its resident warps, so the run time is
+    // ~ the instances placed on the busiest SM (blocks are dealt round-robin),
+    // as long as the occupancy is similar; a ragged tail of 128-wide blocks
+    // costs up to 96 instances more than one of 32-wide blocks.
+    auto busiest = [&](int occ, int block) {
+      if (occ <= 0) return 1e30;
+      const double nb = std::ceil((double)P.n_inst / block);
+      return std::ceil(nb / sms) * block * (1.0 + 0.02 * (8.0 / (occ * block / 32.0)));
     };
-    if (occ128[nc] <= 0 || waves(occ32[nc], 32) < waves(occ128[nc], 128))
+    if (occ128[nc] <= 0 || busiest(occ32[nc], 32) < busiest(occ128[nc], 128))
       return launch_sim<N, M, S, 32>(P, st, tr, k0, K, s);
     return launch_sim<N, M, S, 128>(P, st, tr, k0, K, s);
   }
