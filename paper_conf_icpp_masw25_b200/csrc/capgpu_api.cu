@@ -314,6 +314,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   s.pmin = take(ns);
   s.pmax = take(ns);
   s.s_prev = take((int64_t)h.M * ni);
+  q = (double *)(((uintptr_t)q + 31) & ~(uintptr_t)31);  // 16-byte vector loads of the grid table
   GridEntry *gdev = (GridEntry *)take(4 * (int64_t)n_class * CAPGPU_MAX_LEVELS);
   KnobConst *kdev = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 7) / 8);
   cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice);

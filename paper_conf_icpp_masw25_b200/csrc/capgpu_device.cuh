@@ -349,15 +349,20 @@ __device__ __forceinline__ double solve_block_convex(const KnobConst *kc, const 
   double s = 0.0;
 #pragma unroll 1
   for (int it = 0; it <= N; ++it) {
-    double num = base, den = den_all;
+    // branch-free: 0/1 mask per knob (one FSEL), two partial sums each for ILP
+    double num0 = base, num1 = 0.0, den0 = den_all, den1 = 0.0;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
-      if ((up >> (2 * j + 1)) & 1u) {
-        num += ad[j];
-        den -= cta[j];
+      const double mk = ((up >> (2 * j + 1)) & 1u) ? 1.0 : 0.0;
+      if (j & 1) {
+        num1 = fma(mk, ad[j], num1);
+        den1 = fma(-mk, cta[j], den1);
+      } else {
+        num0 = fma(mk, ad[j], num0);
+        den0 = fma(-mk, cta[j], den0);
       }
     }
-    s = num * rcp_fast(den);
+    s = (num0 + num1) * rcp_fast(den0 + den1);
     uint32_t nu = 0u;
 #pragma unroll
     for (int j = 0; j < N; ++j) nu |= (fma(-ctau[j], s, kc[j].m) > kc[j].hi ? 2u : 0u) << (2 * j);
@@ -422,7 +427,7 @@ __device__ __forceinline__ int level_of(const KnobConst &kc, const GridEntry *ta
   // estimate, then one exact correction each way against the thresholds
   int l = __double2int_rd(fma(v - kc.f_min, kc.inv_step, 0.5));
   l = min(max(l, 0), kc.L - 1);
-  const double2 mm = *reinterpret_cast<const double2 *>(&tab[l].mid_lo);
+  const double2 mm = __ldg(reinterpret_cast<const double2 *>(&tab[l].mid_lo));
   return l + (v > mm.y ? 1 : 0) - (v <= mm.x ? 1 : 0);
 }
 
@@ -444,7 +449,7 @@ __device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const Grid
       const GridEntry *tab = grid + kc.cls * kMaxL;
       const double v = __dadd_rn(u0[j], acc[j]);
       const int l = level_of<N>(kc, tab, v);
-      const double2 lg = *reinterpret_cast<const double2 *>(&tab[l].level);
+      const double2 lg = __ldg(reinterpret_cast<const double2 *>(&tab[l].level));
       acc[j] = __dadd_rn(v, -lg.x);
       fs[j] = __dadd_rn(fs[j], lg.x);
       const double capj = __dmul_rn(thr_max[j], lg.y);

@@ -247,9 +247,7 @@ __global__ void k_identify(DevParams P, StatePtrs st, const double *F_user, cons
 // Per instance: base cap and the virtual period -1 (Q23): u0 = f_min, acc = 0.
 template <int N>
 __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
-  __shared__ GridEntry sgrid[kMaxN * kMaxL];
-  load_grid(P, sgrid);
-  __syncthreads();
+  const GridEntry *sgrid = P.grid;
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= P.n_inst) return;
   const int64_t si = i / P.n_caps;
@@ -415,16 +413,24 @@ struct SlabLayout {
                        oBA = T + 5 * N, oAM = T + 6 * N;
 };
 
+// Resident warps per SM the register allocation must allow: small models get
+// more warps to hide the FP64 latency; N >= 8 is bounded by the slab anyway.
+template <int N>
+struct SimOccupancy {
+  static constexpr int warps = N <= 4 ? 16 : (N <= 6 ? 12 : 8);
+};
+
 template <int N, int M, int S, int BLOCK>
-__global__ void __launch_bounds__(BLOCK) k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
+__global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
+    k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
   using SL = SlabLayout<N>;
   extern __shared__ __align__(16) double smem[];
-  GridEntry *sgrid = reinterpret_cast<GridEntry *>(smem);
-  load_grid(P, sgrid);
-  __syncthreads();
+  // grid tables: read-only global (L1-resident, 1 KB per class) so the whole
+  // shared memory goes to the per-thread slabs
+  const GridEntry *sgrid = P.grid;
   int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x;
   if (i >= P.n_inst) return;
-  double *my = smem + 4 * P.n_class * kMaxL + threadIdx.x * SL::F;
+  double *my = smem + threadIdx.x * SL::F;
   const Slab Sm{my};
   const Slab MU{my + SL::oMU};
   const Slab SF{my + SL::oSFP};
@@ -759,7 +765,7 @@ struct LaunchN {
 // whole per-instance run time).
 template <int N, int M, int S, int BLOCK>
 int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
-  const int smem = (int)(sizeof(double) * (4 * P.n_class * kMaxL + SlabLayout<N>::F * BLOCK));
+  const int smem = (int)(sizeof(double) * SlabLayout<N>::F * BLOCK);
   cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   k_simulate<N, M, S, BLOCK><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
   return (int)cudaGetLastError();
@@ -768,7 +774,8 @@ int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int
 template <int N, int M, int S>
 int sim_occupancy(int block, int n_class) {
   int nb = 0;
-  const int smem_per_block = (int)(sizeof(double) * (4 * n_class * kMaxL + SlabLayout<N>::F * block));
+  (void)n_class;
+  const int smem_per_block = (int)(sizeof(double) * SlabLayout<N>::F * block);
   if (block == 32) {
     cudaFuncSetAttribute(k_simulate<N, M, S, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 32>, 32, smem_per_block);
