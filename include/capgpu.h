@@ -207,6 +207,19 @@ int capgpu_simulate(capgpu_ctx *ctx, int64_t periods, const capgpu_workload *wl,
                     const capgpu_trace *tr, void *stream);
 int capgpu_sim_reset(capgpu_ctx *ctx);
 
+/* Hierarchical budget (wl->hierarchical) for n_ctx shards that live on ONE
+ * device in one process (ranks 0..n_ctx-1 of world n_ctx, created without
+ * NCCL): the contexts step period by period together and the per-period
+ * all-reduce is an in-process (loopback) sum of their zero-padded block
+ * vectors.  Results are bitwise identical to one context holding all servers
+ * and to n_ctx processes over NCCL.  trs: NULL or [n_ctx]. */
+int capgpu_simulate_group(capgpu_ctx **ctxs, int32_t n_ctx, int64_t periods, const capgpu_workload *wl,
+                          const capgpu_trace *const *trs, void *stream);
+
+/* Host copy of the fixed-order pairwise tree the device uses for cluster sums
+ * (zero-pad to 2^m >= n; for h = 2^(m-1)..1: v[i] += v[i+h]). */
+int capgpu_tree_sum_host(const double *v, int64_t n, double *out);
+
 /* Copy the device plant state of the simulation to host-visible buffers for
  * checkpointing / parity checks: fbar, acc, thr [N][n_inst]; p [n_inst]
  * (device pointers, nullable). */

@@ -131,6 +131,11 @@ int ora_simulate(const ora_cfg *c, const ora_workload *w, int n_inst, const int6
                  double *A0_out /*[n_inst][N]*/, int use_definition_mode);
 
 /* ---- S5 hierarchical budget (cfg 4, Q16) */
+int ora_simulate_hier(const ora_cfg *c, const ora_workload *w, int n_servers, int rack, double cluster_frac,
+                      double rack_frac, const double *W_replay, double W0_replay, int n_total, int n_tr,
+                      const int64_t *tr_srv,
+                      double *tr_p, double *tr_cap, double *tr_u, uint32_t *tr_active, uint32_t *tr_tie,
+                      uint8_t *tr_levels, double *agg_W, double *agg_P, double *final_p);
 void ora_budget_caps(int n_servers, int rack, const double *pmin, const double *w, double W,
                      double B_c, double pmin_tot, const double *B_rack_max, double *cap);
 

@@ -112,6 +112,9 @@ def lib():
                                    dp, C.POINTER(OraSummary), dp, C.c_int]
         L.ora_budget_caps.argtypes = [C.c_int, C.c_int, dp, dp, C.c_double, C.c_double,
                                       C.c_double, dp, dp]
+        L.ora_simulate_hier.argtypes = [cp, wp, C.c_int, C.c_int, C.c_double, C.c_double, dp, C.c_double,
+                                        C.c_int, C.c_int, C.POINTER(C.c_int64), dp, dp, dp, u32p, u32p,
+                                        C.POINTER(C.c_uint8), dp, dp, dp]
         _lib = L
     return _lib
 
@@ -336,6 +339,34 @@ class Oracle:
         out["final_p"] = final_p
         out["A0"] = A0
         out["summary"] = summaries_to_numpy(summ, M)
+        return out
+
+    def simulate_hier(self, n_servers, tr_srv, periods=None, W_replay=None, W0_replay=0.0, n_total=None):
+        """cfg 4 hierarchical budget, every server stepping together (Q16).
+        Replay mode (W_replay given): simulate only servers [0, n_servers) of an
+        n_total-server cluster, taking the cluster sums W(k) from W_replay."""
+        wl = self.desc["workload"]
+        w = make_workload(self.desc, periods)
+        K, n, M, S = w.periods, self.n, self.M, self.S
+        tr_srv = np.ascontiguousarray(np.asarray(tr_srv, dtype=np.int64))
+        nt = len(tr_srv)
+        out = dict(p=np.zeros((K, nt)), cap=np.zeros((K, nt)), u=np.zeros((K, nt, M, n)),
+                   active=np.zeros((K, nt, M), dtype=np.uint32), tie=np.zeros((K, nt, M), dtype=np.uint32),
+                   levels=np.zeros((K, nt, S, n), dtype=np.uint8), agg_W=np.zeros(K), agg_P=np.zeros(K),
+                   final_p=np.zeros(n_servers))
+        wr = None if W_replay is None else np.ascontiguousarray(np.asarray(W_replay, dtype=np.float64))
+        u32 = C.POINTER(C.c_uint32)
+        rc = self.L.ora_simulate_hier(C.byref(self.cfg), C.byref(w), n_servers, wl.get("rack", 16),
+                                      wl.get("cluster_frac", 0.55), wl.get("rack_frac", 0.9),
+                                      _dp(wr) if wr is not None else None, float(W0_replay),
+                                      int(n_total if n_total is not None else n_servers), nt,
+                                      tr_srv.ctypes.data_as(C.POINTER(C.c_int64)), _dp(out["p"]), _dp(out["cap"]),
+                                      _dp(out["u"]), out["active"].ctypes.data_as(u32),
+                                      out["tie"].ctypes.data_as(u32),
+                                      out["levels"].ctypes.data_as(C.POINTER(C.c_uint8)), _dp(out["agg_W"]),
+                                      _dp(out["agg_P"]), _dp(out["final_p"]))
+        if rc != 0:
+            raise RuntimeError(f"ora_simulate_hier rc={rc}")
         return out
 
     def budget_caps(self, pmin, w, W, B_c, pmin_tot, B_rack_max, rack):

@@ -71,7 +71,7 @@ SYMBOLS = ["capgpu_version", "capgpu_status_string", "capgpu_last_error", "capgp
            "capgpu_create", "capgpu_destroy", "capgpu_state_bytes", "capgpu_identify", "capgpu_set_prior",
            "capgpu_model_reset", "capgpu_assign_weights", "capgpu_control_step", "capgpu_simulate",
            "capgpu_sim_reset", "capgpu_sim_state", "capgpu_sim_caps", "capgpu_nccl_unique_id", "capgpu_shard_range",
-           "capgpu_debug_gen", "capgpu_fp64_peak"]
+           "capgpu_debug_gen", "capgpu_fp64_peak", "capgpu_simulate_group", "capgpu_tree_sum_host"]
 
 _lib = None
 
@@ -110,6 +110,9 @@ def lib():
     L.capgpu_shard_range.restype = C.c_int64
     L.capgpu_debug_gen.argtypes = [_VP, C.c_int64, C.c_int32, C.c_double, _VP, _VP, _VP, _VP, _VP, _VP]
     L.capgpu_fp64_peak.argtypes = [C.POINTER(C.c_double), _VP]
+    L.capgpu_simulate_group.argtypes = [C.POINTER(_VP), C.c_int32, C.c_int64, C.POINTER(Workload),
+                                        C.POINTER(C.POINTER(Trace)), _VP]
+    L.capgpu_tree_sum_host.argtypes = [C.POINTER(C.c_double), C.c_int64, C.POINTER(C.c_double)]
     _lib = L
     return L
 
@@ -152,6 +155,32 @@ def nccl_unique_id() -> bytes:
     buf = (C.c_uint8 * 128)()
     _check(lib().capgpu_nccl_unique_id(C.byref(buf)))
     return bytes(buf)
+
+
+def simulate_group(ctxs, periods: int, workload, trace_insts=None, summaries: bool = True):
+    """capgpu_simulate_group: several shards of the hierarchical budget on one
+    GPU stepping together with a loopback all-reduce.  Returns one output dict
+    per context (like CapGPU.simulate)."""
+    n = len(ctxs)
+    trs, outs = [], []
+    for q, g in enumerate(ctxs):
+        tr, out = g._trace(periods, workload, None if trace_insts is None else trace_insts[q], summaries)
+        trs.append(tr)
+        outs.append(out)
+    arr = (_VP * n)(*[g._ctx for g in ctxs])
+    tptr = (C.POINTER(Trace) * n)(*[C.pointer(t) for t in trs])
+    rc = lib().capgpu_simulate_group(arr, n, periods, C.byref(workload), tptr, _stream())
+    _check(rc, ctxs[0]._ctx)
+    return outs
+
+
+def tree_sum_host(v) -> float:
+    """The library's fixed-order pairwise tree (host copy of the device tree)."""
+    import numpy as np
+    a = np.ascontiguousarray(np.asarray(v, dtype=np.float64))
+    out = C.c_double(0)
+    _check(lib().capgpu_tree_sum_host(a.ctypes.data_as(C.POINTER(C.c_double)), a.size, C.byref(out)))
+    return float(out.value)
 
 
 def fp64_peak_tflops() -> float:
@@ -277,6 +306,12 @@ class CapGPU:
 
     def simulate(self, periods: int, workload: Workload, trace_inst=None, summaries: bool = True,
                  traces=("p", "cap", "u", "ahat", "theta", "active", "rank", "levels", "status"), out=None):
+        tr, out = self._trace(periods, workload, trace_inst, summaries, traces, out)
+        _check(self.L.capgpu_simulate(self._ctx, periods, C.byref(workload), C.byref(tr), _stream()), self._ctx)
+        return out
+
+    def _trace(self, periods, workload, trace_inst=None, summaries=True,
+               traces=("p", "cap", "u", "ahat", "theta", "active", "rank", "levels", "status"), out=None):
         ni, N, M, S = self.n_inst, self.N, self.M, self.S
         tr = Trace()
         if out is None:
@@ -303,8 +338,7 @@ class CapGPU:
         if workload.hierarchical:
             out["agg_W"], out["agg_P"] = self._z(periods), self._z(periods)
             tr.agg_W_d, tr.agg_P_d = _ptr(out["agg_W"]).value, _ptr(out["agg_P"]).value
-        _check(self.L.capgpu_simulate(self._ctx, periods, C.byref(workload), C.byref(tr), _stream()), self._ctx)
-        return out
+        return tr, out
 
     def sim_reset(self):
         _check(self.L.capgpu_sim_reset(self._ctx), self._ctx)

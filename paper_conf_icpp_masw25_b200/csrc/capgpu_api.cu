@@ -457,6 +457,7 @@ __global__ void k_trace_slots_set(int32_t *slot, int64_t n, const int64_t *inst,
 int capgpu_sim_reset(capgpu_ctx *c) {
   if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
   c->sim_ready = false;
+  c->budget.ready = false;
   c->k_global = 0;
   return CAPGPU_OK;
 }
@@ -473,17 +474,19 @@ static void apply_workload(DevParams &d, const capgpu_workload &w) {
   d.cap_mult = w.cap_mult;
 }
 
-int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, const capgpu_trace *tr,
-                    void *stream) {
-  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
-  if (!wl) return fail(c, CAPGPU_E_INVALID, "workload is NULL");
-  if (periods < 1 || periods > (1ll << 30)) return fail(c, CAPGPU_E_INVALID, "periods out of range");
+}  // extern "C"
+
+// Validation of workload + trace, first-call initialisation (plant, S0 sweep,
+// virtual period -1), base-cap override and trace slots.  Nothing is launched
+// before all arguments are validated.
+static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_trace *tr, TracePtrs &t,
+                       cudaStream_t s) {
+  t = TracePtrs{};
   if (wl->demand_kind != 0 && wl->demand_kind != 1) return fail(c, CAPGPU_E_INVALID, "demand_kind");
   if (wl->cap_period < 0 || (wl->cap_period > 0 && !(wl->cap_lo >= 0 && wl->cap_lo <= wl->cap_hi)))
     return fail(c, CAPGPU_E_INVALID, "cap schedule");
   if (wl->hierarchical && c->prm.caps_per_server != 1)
     return fail(c, CAPGPU_E_INVALID, "hierarchical budget needs caps_per_server == 1");
-  TracePtrs t{};
   if (tr) {
     OPT_DEV(c, tr->sum_p_d);
     OPT_DEV(c, tr->sumsq_p_d);
@@ -505,7 +508,6 @@ int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, c
       OPT_DEV(c, tr->rank_d);
       OPT_DEV(c, tr->levels_d);
       OPT_DEV(c, tr->status_d);
-      if (periods > (1ll << 24)) return fail(c, CAPGPU_E_INVALID, "traced runs are limited to 2^24 periods");
     }
     OPT_DEV(c, tr->agg_W_d);
     OPT_DEV(c, tr->agg_P_d);
@@ -528,7 +530,7 @@ int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, c
     t.rank = tr->rank_d;
     t.levels = tr->levels_d;
   }
-  cudaStream_t s = (cudaStream_t)stream;
+  if (wl->cap_base_d) NEED_DEV(c, wl->cap_base_d);
   apply_workload(c->dp, *wl);
   if (!c->sim_ready) {
     int rc = ensure_servers(c, s);
@@ -543,31 +545,120 @@ int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, c
     c->sim_ready = true;
     c->k_global = 0;
     c->wl = *wl;
-    if (wl->hierarchical) {
-      int rb = budget_setup(c->budget, c->dp, c->st, *wl, c->shard, s, c->err);
-      if (rb) return rb;
-    }
   }
-  if (wl->cap_base_d) {
-    NEED_DEV(c, wl->cap_base_d);
+  if (wl->cap_base_d)
     CK_CUDA(c, cudaMemcpyAsync(c->st.cap_base, wl->cap_base_d, sizeof(double) * c->n_inst,
                                cudaMemcpyDeviceToDevice, s));
-  }
   if (t.n_trace > 0) {
     k_trace_slots<<<grid_for(c->n_inst, 256), 256, 0, s>>>(c->st.trace_slot, c->n_inst, nullptr, 0);
     k_trace_slots_set<<<grid_for(t.n_trace, 256), 256, 0, s>>>(c->st.trace_slot, c->n_inst, tr->trace_inst_d,
                                                                t.n_trace);
     CK_CUDA(c, cudaGetLastError());
   }
+  return CAPGPU_OK;
+}
+
+// S5 setup for a set of shards stepping together (1 = this process only,
+// NCCL if world > 1; n > 1 = loopback shards on one GPU): allocation, w_i(0),
+// cluster constants (Pmin_tot, Pmax_tot -> B_c) and W(0), all through the
+// same deterministic block-sum / all-reduce / tree path as every period.
+static int budget_setup_group(capgpu_ctx **cs, int n, const capgpu_workload &wl, cudaStream_t s) {
+  Budget *bs[64];
+  for (int q = 0; q < n; ++q) {
+    capgpu_ctx *c = cs[q];
+    bs[q] = &c->budget;
+    if (c->prm.caps_per_server != 1) return fail(c, CAPGPU_E_INVALID, "hierarchical budget needs caps_per_server == 1");
+    int rc = budget_alloc(c->budget, c->dp, wl, c->shard, c->err);
+    if (!rc) rc = budget_setup_local(c->budget, c->dp, c->st, c->L, s, c->err);
+    if (rc) return rc;
+  }
+  int rc = budget_reduce(bs, n, true, s, cs[0]->err);
+  for (int q = 0; q < n && !rc; ++q) rc = budget_tree(*bs[q], nullptr, nullptr, 0, s, cs[q]->err);
+  for (int q = 0; q < n && !rc; ++q) rc = budget_finish_setup(*bs[q], s, cs[q]->err);
+  if (!rc) rc = budget_reduce(bs, n, false, s, cs[0]->err);
+  for (int q = 0; q < n && !rc; ++q) rc = budget_tree(*bs[q], nullptr, nullptr, 0, s, cs[q]->err);
+  if (rc) return rc;
+  for (int q = 0; q < n; ++q) bs[q]->ready = true;
+  return CAPGPU_OK;
+}
+
+extern "C" {
+
+int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, const capgpu_trace *tr,
+                    void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  if (!wl) return fail(c, CAPGPU_E_INVALID, "workload is NULL");
+  if (periods < 1 || periods > (1ll << 30)) return fail(c, CAPGPU_E_INVALID, "periods out of range");
+  if (tr && tr->n_trace > 0 && periods > (1ll << 24))
+    return fail(c, CAPGPU_E_INVALID, "traced runs are limited to 2^24 periods");
+  if (wl->hierarchical && c->shard.world > 1 && !c->budget.comm)
+    return fail(c, CAPGPU_E_INVALID, "world > 1 hierarchical runs need NCCL (shard.use_nccl) or capgpu_simulate_group");
+  TracePtrs t;
+  cudaStream_t s = (cudaStream_t)stream;
+  int rc = sim_prepare(c, wl, tr, t, s);
+  if (rc) return rc;
   if (wl->hierarchical) {
-    int rc = budget_simulate(c->budget, c->dp, c->st, t, c->L, c->k_global, periods, tr ? tr->agg_W_d : nullptr,
-                             tr ? tr->agg_P_d : nullptr, s, c->err);
+    if (!c->budget.ready) {
+      capgpu_ctx *cs[1] = {c};
+      rc = budget_setup_group(cs, 1, *wl, s);
+      if (rc) return rc;
+    }
+    rc = budget_simulate(c->budget, c->dp, c->st, t, c->L, c->k_global, periods, tr ? tr->agg_W_d : nullptr,
+                         tr ? tr->agg_P_d : nullptr, s, c->err);
     if (rc) return rc;
   } else {
     int e = c->L.simulate(c->dp, c->st, t, c->k_global, (int)periods, s);
     if (e) return cuda_fail(c, (cudaError_t)e, "simulate");
   }
   c->k_global += periods;
+  return CAPGPU_OK;
+}
+
+int capgpu_simulate_group(capgpu_ctx **ctxs, int32_t n_ctx, int64_t periods, const capgpu_workload *wl,
+                          const capgpu_trace *const *trs, void *stream) {
+  if (!ctxs || n_ctx < 1 || n_ctx > 64) return fail(nullptr, CAPGPU_E_INVALID, "bad context list");
+  if (!wl || !wl->hierarchical) return fail(nullptr, CAPGPU_E_INVALID, "group simulation is for the hierarchical budget");
+  if (periods < 1 || periods > (1ll << 30)) return fail(nullptr, CAPGPU_E_INVALID, "periods out of range");
+  for (int q = 0; q < n_ctx; ++q) {
+    capgpu_ctx *c = ctxs[q];
+    if (!c) return fail(nullptr, CAPGPU_E_INVALID, "NULL context in group");
+    if (c->shard.world != n_ctx || c->shard.rank != q || c->budget.comm)
+      return fail(c, CAPGPU_E_INVALID, "group member %d must be rank %d of world %d without NCCL", q, q, n_ctx);
+    if (c->N != ctxs[0]->N || c->M != ctxs[0]->M || c->shard.n_servers_global != ctxs[0]->shard.n_servers_global)
+      return fail(c, CAPGPU_E_INVALID, "group members must share N, M and the global server count");
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  TracePtrs t[64];
+  for (int q = 0; q < n_ctx; ++q) {
+    capgpu_ctx *c = ctxs[q];
+    if (c->wl.hierarchical && c->sim_ready && c->k_global != ctxs[0]->k_global)
+      return fail(c, CAPGPU_E_ORDER, "group members are out of step");
+    int rc = sim_prepare(c, wl, trs ? trs[q] : nullptr, t[q], s);
+    if (rc) return rc;
+  }
+  if (!ctxs[0]->budget.ready) {
+    int rc = budget_setup_group(ctxs, n_ctx, *wl, s);
+    if (rc) return rc;
+  }
+  Budget *bs[64];
+  for (int q = 0; q < n_ctx; ++q) bs[q] = &ctxs[q]->budget;
+  const int64_t k0 = ctxs[0]->k_global;
+  for (int64_t kk = 0; kk < periods; ++kk) {
+    for (int q = 0; q < n_ctx; ++q) {
+      capgpu_ctx *c = ctxs[q];
+      int rc = budget_period_local(c->budget, c->dp, c->st, t[q], c->L, k0 + kk, (int)kk, (int)periods, s, c->err);
+      if (rc) return rc;
+    }
+    int rc = budget_reduce(bs, n_ctx, false, s, ctxs[0]->err);
+    if (rc) return rc;
+    for (int q = 0; q < n_ctx; ++q) {
+      const capgpu_trace *tq = trs ? trs[q] : nullptr;
+      rc = budget_tree(ctxs[q]->budget, tq ? tq->agg_W_d : nullptr, tq ? tq->agg_P_d : nullptr, (int)kk, s,
+                       ctxs[q]->err);
+      if (rc) return rc;
+    }
+  }
+  for (int q = 0; q < n_ctx; ++q) ctxs[q]->k_global += periods;
   return CAPGPU_OK;
 }
 

