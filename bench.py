@@ -54,6 +54,25 @@ def fp64_peak_derived() -> float:
     return B200_SMS * FP64_FMA_PER_CLK_PER_SM * 2 * SM_MAX_MHZ * 1e6 / 1e12
 
 
+def period_bytes(N: int, M: int) -> int:
+    """Algorithmic HBM bytes per server-step in per-period mode (cfg 4): the
+    mutable state read + written once per period (fbar, acc, thr, mu_f, Sfp,
+    Sigma, w, mu_p, p, w_i, warm starts) and the read-only constants read once
+    (A0, a_true, thr_max, base, amp, C, pmin, pmax)."""
+    T = N * (N + 1) // 2
+    rw = 8 * (5 * N + T + 4) + 12 * M
+    ro = 8 * (5 * N + 3)
+    return 2 * rw + ro
+
+
+def measured_hbm_gbs() -> float:
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            return float(json.load(fh)["hbm_gbs"])
+    except Exception:
+        return 6650.0  # fallback of /opt/skills/guides/B200_PROFILING.md
+
+
 # ---------------------------------------------------------------- clocks
 
 REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
@@ -142,7 +161,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3, 5])
+    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3, 4, 5])
     ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -203,10 +222,29 @@ def main():
 
     d = configs.get(args.config)
     periods = args.periods or d["periods"]
-    n_srv = d["n_servers"]
     N, M, S = d["n_gpus"] + 1, d["M"], d["controller"]["substeps"]
-    g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=rank * n_srv, world=world, rank=rank,
-                           n_servers_global=world * n_srv)
+    hier = bool(d["workload"].get("hierarchical", False))
+    if hier:
+        # cfg 4: one global cluster sharded over the GPUs (strong scaling); the
+        # per-period cluster aggregate crosses GPUs through NCCL (NVLink).
+        n_global = d["n_servers"]
+        begin, n_srv = G.shard_range(n_global, world, rank, 1024)
+        nccl_id = None
+        if world > 1:
+            uid = torch.zeros(128, dtype=torch.uint8, device=dev)
+            if rank == 0:
+                uid = torch.tensor(list(G.nccl_unique_id()), dtype=torch.uint8, device=dev)
+            dist.broadcast(uid, 0)
+            nccl_id = bytes(uid.cpu().tolist())
+        g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=begin, world=world, rank=rank,
+                               n_servers_global=n_global, nccl_id=nccl_id)
+    else:
+        # cfgs 1-3, 5: independent servers; every rank runs its own shard of the
+        # configuration (weak scaling, no data-path collective)
+        n_srv = d["n_servers"]
+        n_global = world * n_srv
+        g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=rank * n_srv, world=world, rank=rank,
+                               n_servers_global=n_global)
     wl = workload_from(d)
     n_inst = g.n_inst
     stream = torch.cuda.current_stream()
@@ -243,12 +281,14 @@ def main():
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     t_max = float(tt.item())
     steps_per_call = n_inst * periods
-    value = world * steps_per_call * args.steps / t_max
+    total_per_step = (n_global if hier else world * n_inst) * periods
+    value = total_per_step * args.steps / t_max
 
     # ---- e2e through the public API with host buffers: H2D of the per-instance
-    # set points from pinned memory, capgpu_simulate, D2H of the summaries.
-    caps_host = g.sim_caps().cpu().pin_memory()
-    caps_dev = torch.empty_like(caps_host, device=dev)
+    # set points from pinned memory (not for cfg 4: its caps come from the
+    # budget), capgpu_simulate, D2H of the per-instance summaries.
+    caps_host = None if hier else g.sim_caps().cpu().pin_memory()
+    caps_dev = None if hier else torch.empty_like(caps_host, device=dev)
     outs_host = {k: torch.empty(n_inst, dtype=dt, pin_memory=True)
                  for k, dt in (("sum_p", torch.float64), ("max_p", torch.float64), ("n_viol", torch.int32))}
     e2e_evs = []
@@ -256,8 +296,9 @@ def main():
         flush.zero_()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        caps_dev.copy_(caps_host, non_blocking=True)
-        wl.cap_base_d = caps_dev.data_ptr()
+        if not hier:
+            caps_dev.copy_(caps_host, non_blocking=True)
+            wl.cap_base_d = caps_dev.data_ptr()
         out = g.simulate(periods, wl, out=bufs)
         for k in outs_host:
             outs_host[k].copy_(out[k], non_blocking=True)
@@ -269,12 +310,18 @@ def main():
     te = torch.tensor([t_e2e], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_value = world * steps_per_call * len(e2e_evs) / float(te.item())
+    e2e_value = total_per_step * len(e2e_evs) / float(te.item())
 
     flops = algorithmic_flops(N, M, S)
     launch_s = t_local / args.steps
-    achieved = flops * steps_per_call / launch_s / 1e12
-    peak = fp64_peak_derived()
+    if hier:
+        # per-period mode: the state streams through HBM every period
+        bpp = period_bytes(N, M)
+        achieved = bpp * steps_per_call / launch_s / 1e9
+        peak = measured_hbm_gbs()
+    else:
+        achieved = flops * steps_per_call / launch_s / 1e12
+        peak = fp64_peak_derived()
     measured_peak = G.fp64_peak_tflops()
     traffic = None
     prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}_summary.json")
@@ -287,25 +334,39 @@ def main():
             traffic = None
 
     if rank == 0:
+        if hier:
+            roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                    "traffic": traffic, "bytes_per_step": period_bytes(N, M),
+                    "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)",
+                    "note": "per-step time includes the block-sum/tree kernels and the NCCL all-reduce"}
+            mode = "per-period kernels k_period + block sums + all-reduce + fixed-order tree (3 launches/period)"
+            par = f"dp{world} (contiguous 1024-aligned server shards; NCCL all-reduce of 16 KB per period)"
+            launches = 3 * periods * args.steps
+        else:
+            roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                    "frac": achieved / peak, "traffic": traffic, "flops_per_step": flops,
+                    "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 x 1965 MHz "
+                                   "(DESIGN.md §8); measured DFMA microbench in peak_measured",
+                    "peak_measured": measured_peak,
+                    "state_bytes_per_step": state_bytes_per_instance(N, M) / periods}
+            mode = "fused multi-period kernel k_simulate (1 launch per step)"
+            par = f"dp{world} (server shards, no data-path collective)"
+            launches = args.steps
         line = {"metric": "server-control-steps/sec", "value": value, "unit": "server-control-steps/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-                "ms_per_step": 1e3 * t_max / args.steps, "higher_is_better": True, "scaling": "weak",
+                "ms_per_step": 1e3 * t_max / args.steps, "higher_is_better": True,
+                "scaling": "strong" if hier else "weak",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded generator, DESIGN.md §3)",
                 "config": {"workload": workload_name(d, periods), "instances_per_gpu": n_inst,
                            "periods_per_step": periods, "n_knobs": N, "P": d["P"], "M": M, "substeps": S,
-                           "mode": "fused multi-period kernel k_simulate (1 launch per step)",
+                           "mode": mode,
                            "l2": "flushed between timed steps (256 MiB write outside the events)",
-                           "parallelism": f"dp{world} (server shards, no data-path collective)"},
-                "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                             "frac": achieved / peak, "traffic": traffic,
-                             "flops_per_step": flops,
-                             "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 x 1965 MHz "
-                                            "(DESIGN.md §8); measured DFMA microbench in peak_measured",
-                             "peak_measured": measured_peak,
-                             "state_bytes_per_step": state_bytes_per_instance(N, M) / periods},
-                "e2e": {"value": e2e_value, "unit": "server-control-steps/s", "h2d_bytes_per_step": 8 * n_inst,
+                           "parallelism": par},
+                "roofline": roof,
+                "e2e": {"value": e2e_value, "unit": "server-control-steps/s",
+                        "h2d_bytes_per_step": 0 if hier else 8 * n_inst,
                         "d2h_bytes_per_step": 20 * n_inst},
-                "gpu_launches": args.steps,
+                "gpu_launches": launches,
                 "clocks": clocks}
         if world == 1 and not args.no_cpu_baseline:
             rate, sample, cores, _ = oracle_rate(args.config, periods, args.cpu_budget, os.cpu_count() or 1)
