@@ -246,6 +246,11 @@ int capgpu_debug_gen(capgpu_ctx *ctx, int64_t k, int32_t demand_kind, double dem
                      double *a_true_d, double *thr_max_d, double *c_true_d, double *dem_d,
                      double *noise_d, void *stream);
 
+/* Profiling hook: per-instance cycle counters [8][n_inst] (int64, device,
+ * accumulated, caller zeroes) of the fused kernel's phases; only libraries
+ * built with -DCAPGPU_PHASE_TIMING write them.  NULL disables. */
+int capgpu_debug_phase_counters(capgpu_ctx *ctx, long long *counters_d);
+
 /* Microbenchmark: FP64 DFMA throughput of this device (TFLOP/s), for the
  * roofline denominator. */
 int capgpu_fp64_peak(double *tflops_out, void *stream);

@@ -51,12 +51,18 @@ def _deps():
                                                       os.path.join(ROOT, "gen", "capgpu_gen.h")])
 
 
-def _compile(src: str, force: bool, verbose: bool) -> str:
-    obj = os.path.join(BUILD, os.path.basename(src).replace(".cu", ".o"))
+VARIANTS = {
+    # profiling build: per-phase cycle counters in the fused kernel (never the product library)
+    "timing": (["-DCAPGPU_PHASE_TIMING"], "_build_timing", "libcapgpu_timing.so"),
+}
+
+
+def _compile(src: str, force: bool, verbose: bool, bdir: str = BUILD, extra=()) -> str:
+    obj = os.path.join(bdir, os.path.basename(src).replace(".cu", ".o"))
     newest_dep = max(os.path.getmtime(d) for d in _deps() + [src])
     if not force and os.path.exists(obj) and os.path.getmtime(obj) >= newest_dep:
         return obj
-    cmd = [NVCC, *cflags(), "-c", src, "-o", obj]
+    cmd = [NVCC, *cflags(), *extra, "-c", src, "-o", obj]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -68,22 +74,27 @@ def _compile(src: str, force: bool, verbose: bool) -> str:
     return obj
 
 
-def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, jobs: int | None = None, variant: str | None = None) -> str:
+    extra, bdir, lib = ((), BUILD, LIB)
+    if variant:
+        flags, sub, name = VARIANTS[variant]
+        extra, bdir, lib = (flags, os.path.join(PKG, sub), os.path.join(PKG, name))
+    os.makedirs(bdir, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
     jobs = jobs or max(1, min(len(srcs), os.cpu_count() or 4))
     with cf.ThreadPoolExecutor(jobs) as ex:
-        objs = list(ex.map(lambda s: _compile(s, force, verbose), srcs))
+        objs = list(ex.map(lambda s: _compile(s, force, verbose, bdir, extra), srcs))
     newest = max(os.path.getmtime(o) for o in objs)
-    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < newest:
+    if force or not os.path.exists(lib) or os.path.getmtime(lib) < newest:
         _, libdir = nccl_dirs()
-        cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-cudart", "static", f"-L{libdir}", "-l:libnccl.so.2",
+        cmd = [NVCC, *ARCH, "-shared", "-o", lib, *objs, "-cudart", "static", f"-L{libdir}", "-l:libnccl.so.2",
                "-Xlinker", f"-rpath,{libdir}"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr[-8000:]}")
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    var = next((a.split("=", 1)[1] for a in sys.argv if a.startswith("--variant=")), None)
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, variant=var))

@@ -71,7 +71,8 @@ SYMBOLS = ["capgpu_version", "capgpu_status_string", "capgpu_last_error", "capgp
            "capgpu_create", "capgpu_destroy", "capgpu_state_bytes", "capgpu_identify", "capgpu_set_prior",
            "capgpu_model_reset", "capgpu_assign_weights", "capgpu_control_step", "capgpu_simulate",
            "capgpu_sim_reset", "capgpu_sim_state", "capgpu_sim_caps", "capgpu_nccl_unique_id", "capgpu_shard_range",
-           "capgpu_debug_gen", "capgpu_fp64_peak", "capgpu_simulate_group", "capgpu_tree_sum_host"]
+           "capgpu_debug_gen", "capgpu_fp64_peak", "capgpu_simulate_group", "capgpu_tree_sum_host",
+           "capgpu_debug_phase_counters"]
 
 _lib = None
 
@@ -81,10 +82,13 @@ def lib():
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(LIB_PATH):
-        raise RuntimeError(f"{LIB_PATH} missing: run `python -m paper_conf_icpp_masw25_b200.build` "
+    path = LIB_PATH
+    if os.environ.get("CAPGPU_LIB_VARIANT") == "timing":  # profiling build (tools/phase_timing.py)
+        path = os.path.join(_PKG, "libcapgpu_timing.so")
+    if not os.path.exists(path):
+        raise RuntimeError(f"{path} missing: run `python -m paper_conf_icpp_masw25_b200.build` "
                            "(there is no CPU fallback)")
-    L = C.CDLL(LIB_PATH)
+    L = C.CDLL(path)
     L.capgpu_version.restype = C.c_char_p
     L.capgpu_status_string.restype = C.c_char_p
     L.capgpu_status_string.argtypes = [C.c_int]
@@ -113,6 +117,7 @@ def lib():
     L.capgpu_simulate_group.argtypes = [C.POINTER(_VP), C.c_int32, C.c_int64, C.POINTER(Workload),
                                         C.POINTER(C.POINTER(Trace)), _VP]
     L.capgpu_tree_sum_host.argtypes = [C.POINTER(C.c_double), C.c_int64, C.POINTER(C.c_double)]
+    L.capgpu_debug_phase_counters.argtypes = [_VP, _VP]
     _lib = L
     return L
 

@@ -717,6 +717,13 @@ __global__ void k_dfma_peak(double *out, int iters, double a, double b) {
   if (s == 12345.678) out[0] = s;
 }
 
+int capgpu_debug_phase_counters(capgpu_ctx *c, long long *counters_d) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  OPT_DEV(c, counters_d);
+  c->dp.phase = counters_d;
+  return CAPGPU_OK;
+}
+
 int capgpu_fp64_peak(double *tflops_out, void *stream) {
   if (!tflops_out) return fail(nullptr, CAPGPU_E_INVALID, "out is NULL");
   cudaStream_t s = (cudaStream_t)stream;

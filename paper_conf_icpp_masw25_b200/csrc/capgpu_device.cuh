@@ -76,10 +76,31 @@ struct DevParams {
   int64_t n_srv, n_inst;     // local counts
   const GridEntry *grid;     // device [n_class][kMaxL]
   const KnobConst *k_dev;    // device copy of k[] for out-of-line code (keeps P in the param bank)
+  long long *phase;          // [8][n_inst] cycle counters (builds with -DCAPGPU_PHASE_TIMING only)
   KnobConst k[kMaxN];
 };
 
 // ------------------------------------------------------------------ helpers
+
+// Phase timing (profiling builds only): CAPGPU_MARK(P, id, i) adds the cycles
+// since the previous mark to counter `id` of instance i.
+#ifdef CAPGPU_PHASE_TIMING
+struct PhaseClock {
+  long long t;
+};
+#define CAPGPU_PHASE_DECL PhaseClock ph_clk{clock64()};
+#define CAPGPU_MARK(P, id, i)                                                        \
+  do {                                                                               \
+    const long long t_ = clock64();                                                  \
+    if ((P).phase) (P).phase[(int64_t)(id) * (P).n_inst + (i)] += t_ - ph_clk.t;     \
+    ph_clk.t = clock64();                                                            \
+  } while (0)
+#else
+#define CAPGPU_PHASE_DECL
+#define CAPGPU_MARK(P, id, i) \
+  do {                        \
+  } while (0)
+#endif
 
 __device__ __forceinline__ double rcp_fast(double x) {
   // MUFU.RCP64H seed + two Newton steps: ~1 ulp (continuous quantities only).
@@ -371,6 +392,82 @@ __device__ __forceinline__ double solve_block_convex(const KnobConst *kc, const 
   }
   code = up;
   return s;
+}
+
+// All M blocks of the convex case at once (same structure as
+// solve_block_convex).  Shared across blocks: base = beta + a.lo (the
+// all-low test does not depend on c_t), ta_j = tau_j a_j with TA = sum ta_j,
+// ad_j = a_j (h_j - m_j), and the upper thresholds b_j = -(h_j - m_j)/tau_j:
+//   knob j is at its upper bound  <=>  m_j - c tau_j s > h_j  <=>  c s < b_j.
+// Per block and step: s_U = (base + sum_U ad_j) / (1 + c (TA - sum_U ta_j)).
+// The blocks iterate in lock-step (independent dependency chains interleave).
+// act: in = last period's codes (warm start), out = upper codes at the roots.
+template <int N, int M>
+__device__ __forceinline__ void solve_blocks_convex(const DevParams &P, const double (&a)[N], const double (&tau)[N],
+                                                    double base, uint32_t (&act)[M], double (&s)[M]) {
+  if (!(base < 0.0)) {  // root s* = base >= 0 in every block: all knobs at lo
+    uint32_t c = 0u;
+#pragma unroll
+    for (int j = 0; j < N; ++j) c |= (base > 0.0 && tau[j] > 0.0 ? 1u : 0u) << (2 * j);
+#pragma unroll
+    for (int t = 0; t < M; ++t) {
+      s[t] = base;
+      act[t] = c;
+    }
+    return;
+  }
+  double ta[N], ad[N], b[N], TA0 = 0.0, TA1 = 0.0;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    ta[j] = tau[j] * a[j];
+    ad[j] = a[j] * P.k[j].span;
+    b[j] = -P.k[j].span * rcp_fast(tau[j]);  // tau_j = 0 -> -inf: never upper
+    if (j & 1) TA1 += ta[j]; else TA0 += ta[j];
+  }
+  const double TA = TA0 + TA1;
+  uint32_t up[M];
+  bool done[M];
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+    up[t] = act[t] & 0xAAAAAAAAu;
+    done[t] = false;
+    s[t] = 0.0;
+  }
+#pragma unroll 1
+  for (int it = 0; it <= N; ++it) {
+    bool all = true;
+#pragma unroll
+    for (int t = 0; t < M; ++t) {
+      if (done[t]) continue;
+      double n0 = base, n1 = 0.0, d0 = 0.0, d1 = 0.0;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        const double mk = ((up[t] >> (2 * j + 1)) & 1u) ? 1.0 : 0.0;
+        if (j & 1) {
+          n1 = fma(mk, ad[j], n1);
+          d1 = fma(mk, ta[j], d1);
+        } else {
+          n0 = fma(mk, ad[j], n0);
+          d0 = fma(mk, ta[j], d0);
+        }
+      }
+      const double c = P.ct[t];
+      const double st = (n0 + n1) * rcp_fast(fma(c, TA - (d0 + d1), 1.0));
+      const double cs = c * st;
+      uint32_t nu = 0u;
+#pragma unroll
+      for (int j = 0; j < N; ++j) nu |= (cs < b[j] ? 2u : 0u) << (2 * j);
+      s[t] = st;
+      if (nu == up[t]) done[t] = true;
+      else {
+        up[t] = nu;
+        all = false;
+      }
+    }
+    if (all) break;
+  }
+#pragma unroll
+  for (int t = 0; t < M; ++t) act[t] = up[t];
 }
 
 // Solve one block; returns the root s (u and codes follow from it).

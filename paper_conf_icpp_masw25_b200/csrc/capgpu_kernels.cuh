@@ -311,41 +311,50 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double cap
                                                   double &mu_p, SAcc S, VAcc Sfp, A0Acc A0,
                                                   const double (&fbar)[N], double p, TAcc thr, TmAcc thr_max,
                                                   double (&s_prev)[M], uint32_t (&act)[M], double (&u0)[N],
-                                                  uint32_t &status, const InstantOut &out) {
+                                                  uint32_t &status, const InstantOut &out, int64_t inst = 0) {
+  (void)inst;
+  CAPGPU_PHASE_DECL
   // S1 (Eq. 5; Q1-Q4)
   double ahat[N];
   model_push<N>(P.lam, w, mu_f, mu_p, S, Sfp, fbar, p);
+  CAPGPU_MARK(P, 1, inst);
   model_solve<N>(P.rho, P.a_lo, P.a_hi, S, Sfp, A0, ahat);
-  // S2: theta (IEEE division), tau_j = ahat_j / R_j = ahat_j theta_j / r0_j
-  double tau[N], tsum = 0.0;
+  CAPGPU_MARK(P, 2, inst);
+  // S2: tau_j = ahat_j / R_j = ahat_j theta_j / r0_j.  theta only
+  // feeds continuous quantities here, so it uses the fast reciprocal; the
+  // reported theta and ranks (integers, bit-exact) use the IEEE division.
+  double tau[N], tsum0 = 0.0, tsum1 = 0.0;
   {
-    double th[N], tr_[N], tm_[N];
+    double tr_[N], tm_[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       tr_[j] = thr.get(j);
       tm_[j] = thr_max.get(j);
+      const double th = pclamp(tr_[j] * rcp_fast(tm_[j]), P.theta_min, 1.0);
+      if (j & 1) tsum1 += th; else tsum0 += th;
+      tau[j] = ahat[j] * th * P.k[j].inv_r0;
     }
-    weights<N>(P.theta_min, tr_, tm_, th);
+    if (out.theta || out.rank) {
+      double th[N];
+      weights<N>(P.theta_min, tr_, tm_, th);
+      if (out.theta) {
 #pragma unroll
-    for (int j = 0; j < N; ++j) {
-      tsum += th[j];
-      tau[j] = ahat[j] * th[j] * P.k[j].inv_r0;
-    }
-    if (out.theta) {
+        for (int j = 0; j < N; ++j) out.theta[j * out.ld] = th[j];
+      }
+      if (out.rank) {
+        int8_t rk[N];
+        ranks<N>(th, rk);
 #pragma unroll
-      for (int j = 0; j < N; ++j) out.theta[j * out.ld] = th[j];
-    }
-    if (out.rank) {
-      int8_t rk[N];
-      ranks<N>(th, rk);
-#pragma unroll
-      for (int j = 0; j < N; ++j) out.rank[j * out.ld] = rk[j];
+        for (int j = 0; j < N; ++j) out.rank[j * out.ld] = rk[j];
+      }
     }
   }
+  const double tsum = tsum0 + tsum1;
   if (out.ahat) {
 #pragma unroll
     for (int j = 0; j < N; ++j) out.ahat[j * out.ld] = ahat[j];
   }
+  CAPGPU_MARK(P, 3, inst);
   // S3 (Eq. 9-10a)
   double beta = p - cap, smin = 0.0, smax = 0.0;
 #pragma unroll
@@ -355,9 +364,33 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double cap
     smax = fma(ahat[j], P.k[j].hi, smax);
   }
   status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
-  // Blocks t = 0..M-1, one loop body (not unrolled: instruction cache); the
-  // per-block registers rotate so the body indexes no array by t.  act[] holds
-  // last period's codes on entry (warm start) and this period's on exit.
+  if (P.convex) {
+    // all M blocks in lock-step (independent chains interleave; one code copy)
+    double s[M];
+    solve_blocks_convex<N, M>(P, ahat, tau, beta + smin, act, s);
+#pragma unroll
+    for (int t = 0; t < M; ++t) s_prev[t] = s[t];
+    double ctau[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) ctau[j] = P.ct[0] * tau[j];
+    act[0] = block_u<N>(P.k, ctau, s[0], u0);
+    if (out.u) {
+#pragma unroll 1
+      for (int t = 0; t < M; ++t) {
+        double u[N];
+#pragma unroll
+        for (int j = 0; j < N; ++j) ctau[j] = P.ct[t] * tau[j];
+        block_u<N>(P.k, ctau, s_prev[t], u);
+#pragma unroll
+        for (int j = 0; j < N; ++j) out.u[(int64_t)(t * N + j) * out.ld] = u[j];
+      }
+    }
+    return tsum * P.inv_N;
+  }
+  // General (non-convex) path: blocks t = 0..M-1, one loop body (not
+  // unrolled: instruction cache); the per-block registers rotate so the body
+  // indexes no array by t.  act[] holds last period's codes on entry (warm
+  // start) and this period's on exit.
   double ad[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) ad[j] = ahat[j] * P.k[j].span;
@@ -488,6 +521,7 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
 #pragma unroll
   for (int t = 0; t < M; ++t) act_cnt[t] = 0;
 
+  CAPGPU_PHASE_DECL
 #pragma unroll 1
   for (int kk = 0; kk < K; ++kk) {
     const int64_t k = k0 + kk;
@@ -502,8 +536,10 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
       io.theta = tr.theta ? tr.theta + (int64_t)kk * N * tr.n_trace + slot : nullptr;
       io.rank = tr.rank ? tr.rank + (int64_t)kk * N * tr.n_trace + slot : nullptr;
     }
+    CAPGPU_MARK(P, 7, i);
     const double tbar = control_instant<N, M>(P, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
-                                              act, u0, status, io);
+                                              act, u0, status, io, i);
+    CAPGPU_MARK(P, 0, i);
     if (slot >= 0) {
       const int64_t b = (int64_t)kk * tr.n_trace + slot;
       if (tr.p) tr.p[b] = p;
@@ -525,6 +561,7 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
 #pragma unroll
     for (int j = 0; j < N; ++j) thr_max[j] = TM.get(j);
     demand_all<N>(P, kjit, k + 1, bmask, thr_max, BA, AM, dem);
+    CAPGPU_MARK(P, 4, i);
     if (slot >= 0 && tr.levels) {
       double u_l[N], a_l[N];
 #pragma unroll
@@ -536,11 +573,13 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
                             tr.n_trace);
     }
     plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+    CAPGPU_MARK(P, 5, i);
     const double noise = gen_noise(knoise, k + 1, P.noise_scale);
     double pw = c_true;
 #pragma unroll
     for (int j = 0; j < N; ++j) pw = fma(AT.get(j), fbar[j], pw);
     p = pw + noise;
+    CAPGPU_MARK(P, 6, i);
     if (kk >= kw) {
       sum_theta += tbar;
       sum_p += p;
