@@ -440,14 +440,37 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double cap
 template <int N>
 struct SlabLayout {
   static constexpr int T = Tri<N>::size;
-  static constexpr int used = T + 7 * N;
+  // Option: keep the read-only constants in global memory (L2-resident, read
+  // with ld.global.nc each period) to shrink the slab.  Measured on cfg 3
+  // (N = 9): 10 warps/SM but 168 registers with spills -> 2.0 vs 4.4 G
+  // steps/s, so it is off.
+  static constexpr bool ro_global = false;
+  static constexpr int used = T + (ro_global ? 2 : 7) * N;
   static constexpr int F = used | 1;  // odd stride: conflict-free 8-byte accesses
   static constexpr int oMU = T, oSFP = T + N, oA0 = T + 2 * N, oAT = T + 3 * N, oTM = T + 4 * N,
                        oBA = T + 5 * N, oAM = T + 6 * N;
 };
 
+// read-only per-server constants in global memory
+struct LdgAcc {
+  const double *p;
+  int64_t ld;
+  __device__ __forceinline__ double get(int t) const { return __ldg(p + (int64_t)t * ld); }
+};
+
+template <bool G>
+struct RoSel {
+  using type = Slab;
+  static __device__ __forceinline__ Slab make(double *slab, const double *, int64_t) { return Slab{slab}; }
+};
+template <>
+struct RoSel<true> {
+  using type = LdgAcc;
+  static __device__ __forceinline__ LdgAcc make(double *, const double *g, int64_t ld) { return LdgAcc{g, ld}; }
+};
+
 // Resident warps per SM the register allocation must allow: small models get
-// more warps to hide the FP64 latency; N >= 8 is bounded by the slab anyway.
+// more warps to hide the FP64 latency.
 template <int N>
 struct SimOccupancy {
   static constexpr int warps = N <= 4 ? 16 : (N <= 6 ? 12 : 8);
@@ -467,15 +490,17 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   const Slab Sm{my};
   const Slab MU{my + SL::oMU};
   const Slab SF{my + SL::oSFP};
-  const Slab A0{my + SL::oA0};
-  const Slab AT{my + SL::oAT};
-  const Slab TM{my + SL::oTM};
-  const Slab BA{my + SL::oBA};
-  const Slab AM{my + SL::oAM};
 
   int64_t si = i / P.n_caps;
   const uint64_t srv = (uint64_t)(P.srv_begin + si);
   int64_t ls = P.n_srv, li = P.n_inst;
+
+  using RS = RoSel<SL::ro_global>;
+  const typename RS::type A0 = RS::make(my + SL::oA0, st.A0 + si, ls);
+  const typename RS::type AT = RS::make(my + SL::oAT, st.a_true + si, ls);
+  const typename RS::type TM = RS::make(my + SL::oTM, st.thr_max + si, ls);
+  const typename RS::type BA = RS::make(my + SL::oBA, st.base + si, ls);
+  const typename RS::type AM = RS::make(my + SL::oAM, st.amp + si, ls);
 
   // ---- stage state into registers / slab
   double fbar[N], acc[N], thr[N];
@@ -486,11 +511,13 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
     thr[j] = st.thr[j * li + i];
     MU.set(j, st.mu_f[j * li + i]);
     SF.set(j, st.Sfp[j * li + i]);
-    A0.set(j, st.A0[j * ls + si]);
-    AT.set(j, st.a_true[j * ls + si]);
-    TM.set(j, st.thr_max[j * ls + si]);
-    BA.set(j, st.base[j * ls + si]);
-    AM.set(j, st.amp[j * ls + si]);
+    if constexpr (!SL::ro_global) {
+      my[SL::oA0 + j] = st.A0[j * ls + si];
+      my[SL::oAT + j] = st.a_true[j * ls + si];
+      my[SL::oTM + j] = st.thr_max[j * ls + si];
+      my[SL::oBA + j] = st.base[j * ls + si];
+      my[SL::oAM + j] = st.amp[j * ls + si];
+    }
   }
 #pragma unroll
   for (int t = 0; t < SL::T; ++t) Sm.set(t, st.S[t * li + i]);
@@ -1029,12 +1056,21 @@ int sim_occupancy(int block, int n_class) {
   int nb = 0;
   (void)n_class;
   const int smem_per_block = (int)(sizeof(double) * SlabLayout<N>::F * block);
+  // a configuration whose slab exceeds the shared memory is simply not
+  // eligible (occupancy 0); clear the probe's error so it cannot leak
+  cudaError_t e;
   if (block == 32) {
-    cudaFuncSetAttribute(k_simulate<N, M, S, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 32>, 32, smem_per_block);
+    e = cudaFuncSetAttribute(k_simulate<N, M, S, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
+    if (e == cudaSuccess)
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 32>, 32, smem_per_block);
   } else {
-    cudaFuncSetAttribute(k_simulate<N, M, S, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 128>, 128, smem_per_block);
+    e = cudaFuncSetAttribute(k_simulate<N, M, S, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
+    if (e == cudaSuccess)
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 128>, 128, smem_per_block);
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    nb = 0;
   }
   return nb;
 }
