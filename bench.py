@@ -123,9 +123,9 @@ class ClockSampler(threading.Thread):
 # ---------------------------------------------------------------- oracle (CPU baseline / reference arm)
 
 def _oracle_worker(args):
-    cfg, insts, periods = args
+    desc, insts, periods = args
     from oracle import oracle as O
-    o = O.oracle_for(cfg)
+    o = O.Oracle(desc)
     t = time.perf_counter()
     o.simulate(insts, periods=periods, traces=False)
     return time.perf_counter() - t
@@ -137,14 +137,14 @@ def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int):
     import multiprocessing as mp
     from oracle import oracle as O
     O.build()
-    desc = configs.get(cfg)
+    desc = configs.by_name(cfg)
     n_inst = desc["n_servers"] * desc["workload"]["n_caps"]
     cal_p = min(periods, 100)
-    t_cal = _oracle_worker((cfg, [0], cal_p))
+    t_cal = _oracle_worker((desc, [0], cal_p))
     per_inst = t_cal / cal_p * periods
     k = max(1, int(budget_s / max(per_inst, 1e-6)))
     stride = max(1, n_inst // (k * cores))
-    jobs = [(cfg, [((w * k + i) * stride) % n_inst for i in range(k)], periods) for w in range(cores)]
+    jobs = [(desc, [((w * k + i) * stride) % n_inst for i in range(k)], periods) for w in range(cores)]
     ctx = mp.get_context("fork")
     t0 = time.perf_counter()
     with ctx.Pool(cores) as pool:
@@ -161,7 +161,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3, 4, 5])
+    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab"])
     ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -170,7 +170,8 @@ def parse():
 
 
 def workload_name(d, periods):
-    return (f"cfg{d['cfg']}: {d['n_servers']:,} servers x {d['workload']['n_caps']} caps, 1 CPU + "
+    label = f"cfg{d['cfg']}" if isinstance(d["cfg"], int) else "stability sweep (NEXT-4, gains as caps)"
+    return (f"{label}: {d['n_servers']:,} servers x {d['workload']['n_caps']} caps, 1 CPU + "
             f"{d['n_gpus']} GPUs (N={d['n_gpus'] + 1}), P/M={d['P']}/{d['M']}, {periods} periods per step")
 
 
@@ -178,7 +179,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    d = configs.get(args.config)
+    d = configs.by_name(args.config)
     periods = args.periods or d["periods"]
     cores = os.cpu_count() or 1
     total_steps, total_t = 0.0, 0.0
@@ -220,7 +221,7 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
 
-    d = configs.get(args.config)
+    d = configs.by_name(args.config)
     periods = args.periods or d["periods"]
     N, M, S = d["n_gpus"] + 1, d["M"], d["controller"]["substeps"]
     hier = bool(d["workload"].get("hierarchical", False))

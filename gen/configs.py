@@ -21,7 +21,7 @@ CONTROLLER = dict(q=1.0, r0=1e-4, theta_min=0.05, lam=0.95, rho=100.0, a_lo=0.25
 
 _BASE_WORKLOAD = dict(n_caps=1, demand_kind=1, demand_frac=0.7, cap_frac0=0.5, cap_frac_rand=0.0,
                       cap_frac_step=0.0, cap_period=0, cap_lo=0, cap_hi=0, cap_mult=1.0,
-                      hierarchical=False)
+                      hierarchical=False, gain_dlo=0.0, gain_step=0.0)
 
 CONFIGS = {
     # 1 server, 1 CPU + 2 GPUs, P/M = 4/2, 200 periods, fixed cap
@@ -42,6 +42,36 @@ CONFIGS = {
     5: dict(n_servers=262144, n_gpus=3, P=8, M=2, periods=2000, seed=5,
             workload=dict(n_caps=32, cap_frac0=0.0, cap_frac_step=1.0 / 32.0)),
 }
+
+
+def stability_sweep(n_servers: int = 64, n_gains: int = 24, g_lo: float = 0.2, g_hi: float = 6.0,
+                    periods: int = 1000, r0: float = 0.1) -> dict:
+    """NEXT-4: batched gain-mismatch sweep of §4.4.  The paper's
+    1 CPU + 3 GPU server, frozen model (ridge -> inf, so Ahat = A0), noiseless
+    plant and identification (A0 = a exactly), all weights 1 (theta_min = 1,
+    R = r0), constant demand; cap column c runs the plant with true gains g_c a,
+    g_c = g_lo + c (g_hi - g_lo)/(n_gains - 1), set point at the middle of the
+    true plant's range (feasible).  The closed form (tests/stability.py)
+    says the loop converges iff g < 2 + 1/(c_0 kappa), kappa = sum_j A0_j^2 / r0;
+    r0 = 0.1 puts c_0 kappa near 1 so the bound differs visibly from 2.  The
+    default grid avoids g = 2 exactly: there the nominal model's reachable
+    maximum a.(f_max - f_min) + beta sits exactly on the set point, a floating
+    tie of the CAP_INFEASIBLE flag (Q28)."""
+    d = get(5, n_servers=n_servers, periods=periods, noise_std=0.0, rho=1e30, theta_min=1.0,
+            a_lo=0.0, a_hi=1e30, r0=r0, P=8, M=2)
+    step = (g_hi - g_lo) / (n_gains - 1)
+    d["workload"].update(n_caps=n_gains, demand_kind=0, demand_frac=0.7, cap_frac0=0.5, cap_frac_rand=0.0,
+                         cap_frac_step=0.0, gain_dlo=g_lo - 1.0, gain_step=step)
+    d["cfg"] = "stability"
+    return d
+
+
+def by_name(name) -> dict:
+    """bench.py --config: "1".."5" (BASELINE.json configs) or "stab" (the NEXT-4
+    gain sweep at bench size: 16,384 servers x 24 gains x 1,000 periods)."""
+    if str(name) == "stab":
+        return stability_sweep(n_servers=16384)
+    return get(int(name))
 
 
 def knobs(n_gpus: int) -> list[dict]:

@@ -113,6 +113,9 @@ typedef struct {
   double rack_frac;          /* B_rack = rack_frac * sum_rack Pmax */
   const double *cap_base_d;  /* nullable device [n_inst]: operator-set base caps P_s (W) for this
                                 call, replacing the generated ones (the step schedule still applies) */
+  double gain_dlo, gain_step; /* gain-mismatch sweep (NEXT-4, §4.4): the plant of cap
+                                 index c has true gains g_c a with g_c = 1 + gain_dlo + c gain_step
+                                 (0, 0 -> the nominal plant) */
 } capgpu_workload;
 
 /* Optional outputs of capgpu_simulate; every pointer may be NULL.

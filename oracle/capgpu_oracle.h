@@ -56,6 +56,7 @@ typedef struct {
   double cap_frac0, cap_frac_rand, cap_frac_step;
   int64_t cap_period, cap_lo, cap_hi; /* step schedule */
   double cap_mult;
+  double gain_dlo, gain_step; /* gain mismatch (NEXT-4): true gains g_c a, g_c = 1 + dlo + c step */
 } ora_workload;
 
 /* per-instance summary over the last 80 % of periods */

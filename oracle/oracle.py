@@ -55,7 +55,7 @@ class OraWorkload(C.Structure):
                 ("demand_frac", C.c_double), ("cap_frac0", C.c_double),
                 ("cap_frac_rand", C.c_double), ("cap_frac_step", C.c_double),
                 ("cap_period", C.c_int64), ("cap_lo", C.c_int64), ("cap_hi", C.c_int64),
-                ("cap_mult", C.c_double)]
+                ("cap_mult", C.c_double), ("gain_dlo", C.c_double), ("gain_step", C.c_double)]
 
 
 class OraSummary(C.Structure):
@@ -156,6 +156,7 @@ def make_workload(desc: dict, periods: int | None = None) -> OraWorkload:
     w.demand_kind, w.demand_frac = wl["demand_kind"], wl["demand_frac"]
     w.cap_frac0, w.cap_frac_rand, w.cap_frac_step = wl["cap_frac0"], wl["cap_frac_rand"], wl["cap_frac_step"]
     w.cap_period, w.cap_lo, w.cap_hi, w.cap_mult = wl["cap_period"], wl["cap_lo"], wl["cap_hi"], wl["cap_mult"]
+    w.gain_dlo, w.gain_step = wl.get("gain_dlo", 0.0), wl.get("gain_step", 0.0)
     return w
 
 

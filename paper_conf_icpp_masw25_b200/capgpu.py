@@ -53,7 +53,8 @@ class Workload(C.Structure):
                 ("cap_frac_rand", C.c_double), ("cap_frac_step", C.c_double), ("cap_period", C.c_int64),
                 ("cap_lo", C.c_int64), ("cap_hi", C.c_int64), ("cap_mult", C.c_double),
                 ("hierarchical", C.c_int32), ("rack", C.c_int32), ("block", C.c_int32),
-                ("cluster_frac", C.c_double), ("rack_frac", C.c_double), ("cap_base_d", _VP)]
+                ("cluster_frac", C.c_double), ("rack_frac", C.c_double), ("cap_base_d", _VP),
+                ("gain_dlo", C.c_double), ("gain_step", C.c_double)]
 
 
 _VP = C.c_void_p
@@ -203,6 +204,7 @@ def workload_from(desc: dict) -> Workload:
     w.hierarchical = int(wl.get("hierarchical", False))
     w.rack, w.block = wl.get("rack", 16), wl.get("block", 1024)
     w.cluster_frac, w.rack_frac = wl.get("cluster_frac", 0.55), wl.get("rack_frac", 0.9)
+    w.gain_dlo, w.gain_step = wl.get("gain_dlo", 0.0), wl.get("gain_step", 0.0)
     return w
 
 

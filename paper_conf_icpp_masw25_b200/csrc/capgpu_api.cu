@@ -472,6 +472,8 @@ static void apply_workload(DevParams &d, const capgpu_workload &w) {
   d.cap_lo = w.cap_lo;
   d.cap_hi = w.cap_hi;
   d.cap_mult = w.cap_mult;
+  d.gain0 = 1.0 + w.gain_dlo;
+  d.gain_step = w.gain_step;
 }
 
 }  // extern "C"
@@ -487,6 +489,10 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
     return fail(c, CAPGPU_E_INVALID, "cap schedule");
   if (wl->hierarchical && c->prm.caps_per_server != 1)
     return fail(c, CAPGPU_E_INVALID, "hierarchical budget needs caps_per_server == 1");
+  if (!std::isfinite(wl->gain_dlo) || !std::isfinite(wl->gain_step))
+    return fail(c, CAPGPU_E_INVALID, "gain_dlo / gain_step must be finite");
+  if (wl->hierarchical && (wl->gain_dlo != 0.0 || wl->gain_step != 0.0))
+    return fail(c, CAPGPU_E_INVALID, "gain mismatch is not supported with the hierarchical budget");
   if (tr) {
     OPT_DEV(c, tr->sum_p_d);
     OPT_DEV(c, tr->sumsq_p_d);

@@ -70,6 +70,7 @@ struct DevParams {
   double inv_N;              // 1/N for the mean-theta summary
   double ct[kMaxM];          // block weights c_t (Q11)
   double cap_frac0, cap_frac_rand, cap_frac_step, cap_mult;
+  double gain0, gain_step;   // plant gain mismatch g_c = gain0 + c * gain_step, gain0 = 1 + gain_dlo (NEXT-4)
   int64_t cap_period, cap_lo, cap_hi;
   uint64_t seed;
   int64_t srv_begin;         // global id of local server 0
@@ -101,6 +102,12 @@ struct PhaseClock {
   do {                        \
   } while (0)
 #endif
+
+// True-gain factor of instance column `cidx` (NEXT-4, "A' = g A"):
+// g = (1 + gain_dlo) + cidx * gain_step, rounded exactly as the oracle (no FMA).
+__device__ __forceinline__ double plant_gain(const DevParams &P, int cidx) {
+  return __dadd_rn(P.gain0, __dmul_rn((double)cidx, P.gain_step));
+}
 
 __device__ __forceinline__ double rcp_fast(double x) {
   // MUFU.RCP64H seed + two Newton steps: ~1 ulp (continuous quantities only).

@@ -270,8 +270,9 @@ __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
   plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
   const double noise = gen_noise(gen_stream_key(P.seed, GEN_TAG_NOISE, srv), 0, P.noise_scale);
   double pw = st.c_true[si];
+  const double gain = plant_gain(P, cidx);
 #pragma unroll
-  for (int j = 0; j < N; ++j) pw = fma(st.a_true[j * ls + si], fbar[j], pw);
+  for (int j = 0; j < N; ++j) pw = fma(__dmul_rn(gain, st.a_true[j * ls + si]), fbar[j], pw);
   st.p[i] = pw + noise;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
@@ -290,7 +291,15 @@ __global__ void k_init_instances(DevParams P, StatePtrs st, int M) {
     st.act[t * li + i] = 0u;
   }
   const double fr = gen_cap_frac(P.seed, srv, cidx, P.cap_frac0, P.cap_frac_rand, P.cap_frac_step);
-  st.cap_base[i] = gen_cap_base(st.pmin[si], st.pmax[si], fr);
+  // cap inside the TRUE plant's range (P:230 feasibility); with gain 1 this is st.pmin/pmax
+  double ga[N], fmn[N], fmx[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    ga[j] = __dmul_rn(gain, st.a_true[j * ls + si]);
+    fmn[j] = P.k[j].f_min;
+    fmx[j] = P.k[j].f_max;
+  }
+  st.cap_base[i] = gen_cap_base(gen_power_at(st.c_true[si], ga, fmn, N), gen_power_at(st.c_true[si], ga, fmx, N), fr);
 }
 
 // ------------------------------------------------------------------ shared step
@@ -494,6 +503,9 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   int64_t si = i / P.n_caps;
   const uint64_t srv = (uint64_t)(P.srv_begin + si);
   int64_t ls = P.n_srv, li = P.n_inst;
+  // the plant gain is folded into the per-instance slab copy of a_true
+  static_assert(!SL::ro_global, "ro_global would bypass the plant gain");
+  const double gain = plant_gain(P, (int)(i - si * P.n_caps));
 
   using RS = RoSel<SL::ro_global>;
   const typename RS::type A0 = RS::make(my + SL::oA0, st.A0 + si, ls);
@@ -513,7 +525,7 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
     SF.set(j, st.Sfp[j * li + i]);
     if constexpr (!SL::ro_global) {
       my[SL::oA0 + j] = st.A0[j * ls + si];
-      my[SL::oAT + j] = st.a_true[j * ls + si];
+      my[SL::oAT + j] = __dmul_rn(gain, st.a_true[j * ls + si]);
       my[SL::oTM + j] = st.thr_max[j * ls + si];
       my[SL::oBA + j] = st.base[j * ls + si];
       my[SL::oAM + j] = st.amp[j * ls + si];
