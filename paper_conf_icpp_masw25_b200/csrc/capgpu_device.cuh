@@ -567,6 +567,50 @@ __device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const Grid
   }
 }
 
+// The same plant for a compile-time sub-step count S (the fused kernel's
+// common case).  The period's input u_j is constant and |acc_j| <= step_j/2
+// (u in [f_min, f_max]), so every sub-step value v = u + acc lies within
+// 1.5 steps of the level l_u estimated for u: its level is l_u - 1, l_u or
+// l_u + 1, decided by the thresholds mid(l_u - 1) and mid(l_u) exactly as
+// level_of decides it.  The three candidate rows are read once per period
+// (independent loads) instead of two dependent table reads per sub-step, and
+// the capacities min(dem, thr_max g) are formed once per candidate.  Knobs
+// outer, sub-steps unrolled: the knobs' serial acc chains interleave.  Same
+// arithmetic, same order as plant_delta_sigma (bit-identical results).
+template <int N, int S>
+__device__ __forceinline__ void plant_delta_sigma_c(const DevParams &P, const GridEntry *grid, const double (&u0)[N],
+                                                    double (&acc)[N], const double (&dem)[N],
+                                                    const double (&thr_max)[N], double (&fbar)[N], double (&thr)[N]) {
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    const KnobConst &kc = P.k[j];
+    const GridEntry *tab = grid + kc.cls * kMaxL;
+    int l = __double2int_rd(fma(u0[j] - kc.f_min, kc.inv_step, 0.5));
+    l = min(max(l, 0), kc.L - 1);
+    const double2 mm = __ldg(reinterpret_cast<const double2 *>(&tab[l].mid_lo));
+    const double2 c0 = __ldg(reinterpret_cast<const double2 *>(&tab[l].level));
+    const double2 cl = __ldg(reinterpret_cast<const double2 *>(&tab[l > 0 ? l - 1 : 0].level));
+    const double2 ch = __ldg(reinterpret_cast<const double2 *>(&tab[l < kc.L - 1 ? l + 1 : l].level));
+    const double d = dem[j], tm = thr_max[j];
+    const double k0 = __dmul_rn(tm, c0.y), kl = __dmul_rn(tm, cl.y), kh = __dmul_rn(tm, ch.y);
+    const double t0 = d < k0 ? d : k0, tl = d < kl ? d : kl, th = d < kh ? d : kh;
+    double a = acc[j], fs = 0.0, ts = 0.0;
+#pragma unroll
+    for (int s = 0; s < S; ++s) {
+      const double v = __dadd_rn(u0[j], a);
+      const bool up = v > mm.y, dn = v <= mm.x;
+      const double lev = up ? ch.x : (dn ? cl.x : c0.x);
+      const double tt = up ? th : (dn ? tl : t0);
+      a = __dadd_rn(v, -lev);
+      fs = __dadd_rn(fs, lev);
+      ts = __dadd_rn(ts, tt);
+    }
+    acc[j] = a;
+    fbar[j] = __dmul_rn(fs, P.inv_S);
+    thr[j] = __dmul_rn(ts, P.inv_S);
+  }
+}
+
 // Trace of the level indices (traced instances only): replays the same
 // delta-sigma from the pre-period accumulators.  Out of line (I-cache).
 template <int N>

@@ -611,7 +611,10 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
       plant_trace_levels<N>(P.k_dev, P.S, sgrid, u_l, a_l, tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot,
                             tr.n_trace);
     }
-    plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+    if constexpr (S > 0)
+      plant_delta_sigma_c<N, S>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+    else
+      plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
     CAPGPU_MARK(P, 5, i);
     const double noise = gen_noise(knoise, k + 1, P.noise_scale);
     double pw = c_true;
@@ -1119,7 +1122,8 @@ struct LaunchNM {
   }
   static int simulate(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K,
                       cudaStream_t s) {
-    return sim_s<0>(P, st, tr, k0, K, s);
+    // S = 4 (every BASELINE config) gets the compile-time sub-step plant
+    return P.S == 4 ? sim_s<4>(P, st, tr, k0, K, s) : sim_s<0>(P, st, tr, k0, K, s);
   }
   static int control_step(const DevParams &P, const StatePtrs &st, const double *p, const double *f,
                           const double *thr, const double *tm, const double *cap, double *u, uint32_t *act,
