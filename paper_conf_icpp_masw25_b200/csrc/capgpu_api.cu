@@ -218,6 +218,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   d.a_floor = prm.a_floor;
   d.noise_scale = prm.noise_std * std::sqrt(3.0);
   d.inv_S = 1.0 / (double)prm.substeps;
+  d.inv_lam = 1.0 / prm.lambda;
   // Q11: c_t = Q for t < M-1, c_{M-1} = (P - M + 1) Q
   for (int t = 0; t < h.M; ++t) d.ct[t] = t < h.M - 1 ? prm.q : (double)(h.P - h.M + 1) * prm.q;
   d.seed = prm.seed;

@@ -65,6 +65,7 @@ struct DevParams {
   int32_t convex;            // 1 iff lo_j == m_j (= f_min) for every knob: phi convex on s <= 0
   double demand_frac;
   double q, theta_min, lam, rho, a_lo, a_hi, a_floor;
+  double inv_lam;             // 1 / lam (scaled Welford state of the fused kernel)
   double noise_scale;        // sigma * sqrt(3) (host-computed)
   double inv_S;              // 1/S, exact (S power of two, Q22)
   double inv_N;              // 1/N for the mean-theta summary
@@ -131,12 +132,18 @@ __device__ __forceinline__ double pclamp(double x, double lo, double hi) {
 // Weighted Welford push (Q1-Q3): w <- lam w + 1, delta = z - mu,
 // mu += delta / w, Sigma <- lam Sigma + (1 - 1/w) delta delta^T
 // (= delta (z - mu_new)^T in exact arithmetic).
-template <int N, class SAcc, class VAcc>
-__device__ __forceinline__ void model_push(double lam, double &w, VAcc mu_f, double &mu_p, SAcc S, VAcc Sfp,
-                                           const double (&f)[N], double p) {
+// Scaled form (fused kernel): the stored Sigma' = Sigma / Lambda with
+// Lambda = lam^k since the start of the call, so the decay needs no multiply:
+// Sigma' <- Sigma' + (e / Lambda_new) delta delta^T (inv_lam_k = 1 / Lambda_new);
+// the solve uses rho / Lambda (same solution), and the caller multiplies
+// Sigma' back by Lambda before it leaves the kernel (and every 1024 periods).
+// SCALED = false: the plain form above (state in HBM, one period per launch).
+template <int N, bool SCALED, class SAcc, class VAcc>
+__device__ __forceinline__ void model_push(double lam, double inv_lam_k, double &w, VAcc mu_f, double &mu_p,
+                                           SAcc S, VAcc Sfp, const double (&f)[N], double p) {
   w = fma(lam, w, 1.0);
   const double iw = rcp_fast(w);
-  const double e = 1.0 - iw;
+  const double e = SCALED ? (1.0 - iw) * inv_lam_k : 1.0 - iw;
   double df[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
@@ -153,9 +160,15 @@ __device__ __forceinline__ void model_push(double lam, double &w, VAcc mu_f, dou
 #pragma unroll
     for (int j = i; j < N; ++j) {
       const int t = Tri<N>::idx(i, j);
-      S.set(t, fma(lam, S.get(t), ei * df[j]));
+      if constexpr (SCALED)
+        S.set(t, fma(ei, df[j], S.get(t)));
+      else
+        S.set(t, fma(lam, S.get(t), ei * df[j]));
     }
-    Sfp.set(i, fma(lam, Sfp.get(i), df[i] * edp));
+    if constexpr (SCALED)
+      Sfp.set(i, fma(df[i], edp, Sfp.get(i)));
+    else
+      Sfp.set(i, fma(lam, Sfp.get(i), df[i] * edp));
   }
 }
 

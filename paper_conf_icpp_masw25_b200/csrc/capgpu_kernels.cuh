@@ -315,8 +315,8 @@ struct InstantOut {
 // roots s_t (warm starts for the next period), the per-block active codes and
 // the status; returns mean_j theta_j.  Only short-lived temporaries are kept
 // in registers (the caller's state lives in the slab / registers it owns).
-template <int N, int M, class SAcc, class VAcc, class A0Acc, class TAcc, class TmAcc>
-__device__ __forceinline__ double control_instant(const DevParams &P, double cap, double &w, VAcc mu_f,
+template <int N, int M, bool SCALED = false, class SAcc, class VAcc, class A0Acc, class TAcc, class TmAcc>
+__device__ __forceinline__ double control_instant(const DevParams &P, double inv_lam_k, double cap, double &w, VAcc mu_f,
                                                   double &mu_p, SAcc S, VAcc Sfp, A0Acc A0,
                                                   const double (&fbar)[N], double p, TAcc thr, TmAcc thr_max,
                                                   double (&s_prev)[M], uint32_t (&act)[M], double (&u0)[N],
@@ -325,9 +325,9 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double cap
   CAPGPU_PHASE_DECL
   // S1 (Eq. 5; Q1-Q4)
   double ahat[N];
-  model_push<N>(P.lam, w, mu_f, mu_p, S, Sfp, fbar, p);
+  model_push<N, SCALED>(P.lam, inv_lam_k, w, mu_f, mu_p, S, Sfp, fbar, p);
   CAPGPU_MARK(P, 1, inst);
-  model_solve<N>(P.rho, P.a_lo, P.a_hi, S, Sfp, A0, ahat);
+  model_solve<N>(SCALED ? P.rho * inv_lam_k : P.rho, P.a_lo, P.a_hi, S, Sfp, A0, ahat);
   CAPGPU_MARK(P, 2, inst);
   // S2: tau_j = ahat_j / R_j = ahat_j theta_j / r0_j.  theta only
   // feeds continuous quantities here, so it uses the fast reciprocal; the
@@ -446,6 +446,14 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double cap
 //   S[T] | mu_f[N] | Sfp[N] | A0[N] | a_true[N] | thr_max[N] | base[N] | amp[N]
 // (the model scatter and the read-only constants; fbar, acc, thr stay in
 // registers next to the LDL^T working set).
+// Sigma' and Sigma'_fp (slab offsets 0 and oSFP) times f: the rare
+// renormalisation of the scaled model state (out of line: I-cache).
+template <int N>
+__device__ __noinline__ void slab_rescale(double *my, int oSFP, double f) {
+  for (int t = 0; t < Tri<N>::size; ++t) my[t] *= f;
+  for (int j = 0; j < N; ++j) my[oSFP + j] *= f;
+}
+
 template <int N>
 struct SlabLayout {
   static constexpr int T = Tri<N>::size;
@@ -482,7 +490,11 @@ struct RoSel<true> {
 // more warps to hide the FP64 latency.
 template <int N>
 struct SimOccupancy {
+#ifdef CAPGPU_SIM_WARPS_OVERRIDE
+  static constexpr int warps = CAPGPU_SIM_WARPS_OVERRIDE;
+#else
   static constexpr int warps = N <= 4 ? 16 : (N <= 6 ? 12 : 8);
+#endif
 };
 
 template <int N, int M, int S, int BLOCK>
@@ -560,11 +572,18 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
 #pragma unroll
   for (int t = 0; t < M; ++t) act_cnt[t] = 0;
 
+  // the slab holds Sigma' = Sigma / lam^kk (model_push SCALED); inv_lam_k = lam^-kk
+  double inv_lam_k = 1.0;
+
   CAPGPU_PHASE_DECL
 #pragma unroll 1
   for (int kk = 0; kk < K; ++kk) {
     const int64_t k = k0 + kk;
     const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
+    if ((kk & 1023) == 1023) {  // keep lam^-kk far from overflow: fold it back into Sigma'
+      slab_rescale<N>(my, SL::oSFP, rcp_fast(inv_lam_k));
+      inv_lam_k = 1.0;
+    }
     double u0[N];
     uint32_t status;
     InstantOut io{};
@@ -576,7 +595,8 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
       io.rank = tr.rank ? tr.rank + (int64_t)kk * N * tr.n_trace + slot : nullptr;
     }
     CAPGPU_MARK(P, 7, i);
-    const double tbar = control_instant<N, M>(P, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
+    inv_lam_k *= P.inv_lam;
+    const double tbar = control_instant<N, M, true>(P, inv_lam_k, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
                                               act, u0, status, io, i);
     CAPGPU_MARK(P, 0, i);
     if (slot >= 0) {
@@ -637,16 +657,17 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   // state addresses here instead of keeping the stage-in ones alive (spilled)
   // across the whole period loop.
   asm volatile("" : "+l"(i), "+l"(li), "+l"(ls), "+l"(si));
+  const double lam_k = rcp_fast(inv_lam_k);  // Sigma = lam^kk Sigma'
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     st.fbar[j * li + i] = fbar[j];
     st.acc[j * li + i] = acc[j];
     st.thr[j * li + i] = thr[j];
     st.mu_f[j * li + i] = MU.get(j);
-    st.Sfp[j * li + i] = SF.get(j);
+    st.Sfp[j * li + i] = SF.get(j) * lam_k;
   }
 #pragma unroll
-  for (int t = 0; t < SL::T; ++t) st.S[t * li + i] = Sm.get(t);
+  for (int t = 0; t < SL::T; ++t) st.S[t * li + i] = Sm.get(t) * lam_k;
   st.p[i] = p;
   st.w[i] = w;
   st.mu_p[i] = mu_p;
@@ -771,7 +792,7 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
     }
     const GlobAcc S{st.S + i, ld};
     double u0[N];
-    tbar = control_instant<N, M>(P, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
+    tbar = control_instant<N, M>(P, 0.0, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
                                  RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
     if (slot >= 0) {
       const int64_t b = (int64_t)kk * tr.n_trace + slot;
@@ -932,7 +953,7 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
   const GlobAcc S{st.S + i, ld};
   double u0[N];
   InstantOut io{u_out + i, ahat_out ? ahat_out + i : nullptr, nullptr, rank_out ? rank_out + i : nullptr, ld};
-  control_instant<N, M>(P, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
+  control_instant<N, M>(P, 0.0, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
                         RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
   st.w[i] = w;
   st.mu_p[i] = mu_p;
