@@ -21,7 +21,14 @@ CONTROLLER = dict(q=1.0, r0=1e-4, theta_min=0.05, lam=0.95, rho=100.0, a_lo=0.25
 
 _BASE_WORKLOAD = dict(n_caps=1, demand_kind=1, demand_frac=0.7, cap_frac0=0.5, cap_frac_rand=0.0,
                       cap_frac_step=0.0, cap_period=0, cap_lo=0, cap_hi=0, cap_mult=1.0,
-                      hierarchical=False, gain_dlo=0.0, gain_step=0.0)
+                      hierarchical=False, gain_dlo=0.0, gain_step=0.0,
+                      slo_period=0, slo_lo=0, slo_hi=0, slo_a=None, slo_b=None)
+
+# NEXT-1 (§6.4): latency SLOs as ratios SLO_j / e_min,j for the three
+# tail levels the paper switches between ("30 %", "50 %", "80 % tail").  The
+# paper's percentiles come from measured latency distributions; these ratios
+# are the synthetic stand-ins (Q29): a higher tail = a looser SLO.
+SLO_TAIL = {30: 1.15, 50: 1.35, 80: 1.6}
 
 CONFIGS = {
     # 1 server, 1 CPU + 2 GPUs, P/M = 4/2, 200 periods, fixed cap
@@ -66,11 +73,32 @@ def stability_sweep(n_servers: int = 64, n_gains: int = 24, g_lo: float = 0.2, g
     return d
 
 
+def slo_schedule(n_servers: int = 64, periods: int = 1000, slo_period: int = 200, slo_lo: int = 14,
+                 slo_hi: int = 114) -> dict:
+    """NEXT-1: time-varying SLOs (§6.4) on the paper's 1 CPU + 3 GPU
+    server (P/M = 8/2, P:264).  Phase A: every GPU task at the 50 %-tail SLO;
+    phase B (k mod slo_period in [slo_lo, slo_hi), the paper switches at period
+    14): GPU 0 tightened to the 30 % tail, GPUs 1-2 relaxed to the 80 % tail.
+    The CPU task has no SLO.  Set points P_min + (0.55 + 0.4 U) dP per
+    server: most servers can meet every SLO, some cannot reach their cap with
+    the raised bounds (CAP_INFEASIBLE).  Bursty demand."""
+    d = get(5, n_servers=n_servers, periods=periods)
+    d["workload"].update(n_caps=1, cap_frac0=0.55, cap_frac_rand=0.4, cap_frac_step=0.0,
+                         slo_period=slo_period, slo_lo=slo_lo, slo_hi=slo_hi,
+                         slo_a=[0.0] + [SLO_TAIL[50]] * 3,
+                         slo_b=[0.0, SLO_TAIL[30], SLO_TAIL[80], SLO_TAIL[80]])
+    d["cfg"] = "slo"
+    return d
+
+
 def by_name(name) -> dict:
-    """bench.py --config: "1".."5" (BASELINE.json configs) or "stab" (the NEXT-4
-    gain sweep at bench size: 16,384 servers x 24 gains x 1,000 periods)."""
+    """bench.py --config: "1".."5" (BASELINE.json configs), "stab" (the NEXT-4
+    gain sweep at bench size: 16,384 servers x 24 gains x 1,000 periods) or
+    "slo" (the NEXT-1 SLO schedule: 1,048,576 servers x 1,000 periods)."""
     if str(name) == "stab":
         return stability_sweep(n_servers=16384)
+    if str(name) == "slo":
+        return slo_schedule(n_servers=1048576)
     return get(int(name))
 
 

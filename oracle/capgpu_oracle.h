@@ -57,6 +57,12 @@ typedef struct {
   int64_t cap_period, cap_lo, cap_hi; /* step schedule */
   double cap_mult;
   double gain_dlo, gain_step; /* gain mismatch (NEXT-4): true gains g_c a, g_c = 1 + dlo + c step */
+  /* SLO schedule (NEXT-1, §6.4; Eq. 10b-c; Q29-Q31): per knob the latency
+   * SLO as a ratio SLO_j / e_min,j (0 = no SLO).  Phase B is in force at instant k
+   * while slo_period > 0 and (k mod slo_period) lies in [slo_lo, slo_hi); phase A
+   * otherwise. */
+  int64_t slo_period, slo_lo, slo_hi;
+  double slo_a[ORA_MAXN], slo_b[ORA_MAXN];
 } ora_workload;
 
 /* per-instance summary over the last 80 % of periods */
@@ -64,6 +70,7 @@ typedef struct {
   double sum_p, sumsq_p, max_p, sum_theta;
   int32_t n_window, n_viol;
   int32_t act_count[ORA_MAXM]; /* periods where block t had >= 1 active bound */
+  int32_t n_miss;              /* SLO deadline misses: sub-steps x knobs below the SLO level (Q31) */
 } ora_summary;
 
 #ifdef __cplusplus
@@ -72,6 +79,16 @@ extern "C" {
 
 /* ---- frequency grid (Q15): level(l) = f_min + l*step, mid(l) = f_min + (l+0.5)*step */
 void ora_levels(const ora_cfg *c, int j, double *level, double *mid, double *g);
+
+/* ---- SLO bound (NEXT-1; Eq. 10b-c, Q14, Q30): the lowest grid level
+ * of knob j whose latency e_min (f_max / level)^gamma meets SLO = ratio * e_min.
+ * Returns its index q (n_levels if even f_max misses: SLO infeasible) and the
+ * continuous bound f_req = f_max ratio^(-1/gamma) in *f_req (nullable). */
+int ora_slo_level(const ora_cfg *c, int j, double ratio, double *f_req);
+/* Lower bounds l_j and SLO level indices q_j at instant k of workload w
+ * (static f_lo combined with the SLO level, Q29); returns status bits
+ * (ORA_ST_SLO_INFEASIBLE when an SLO in force is unreachable). */
+uint32_t ora_slo_bounds(const ora_cfg *c, const ora_workload *w, int64_t k, double *lo, int32_t *q);
 
 /* ---- S0 identification */
 int ora_identify_ls(int n, int rows, const double *F, const double *p, double *A, double *C, double *r2);

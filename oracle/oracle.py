@@ -55,13 +55,15 @@ class OraWorkload(C.Structure):
                 ("demand_frac", C.c_double), ("cap_frac0", C.c_double),
                 ("cap_frac_rand", C.c_double), ("cap_frac_step", C.c_double),
                 ("cap_period", C.c_int64), ("cap_lo", C.c_int64), ("cap_hi", C.c_int64),
-                ("cap_mult", C.c_double), ("gain_dlo", C.c_double), ("gain_step", C.c_double)]
+                ("cap_mult", C.c_double), ("gain_dlo", C.c_double), ("gain_step", C.c_double),
+                ("slo_period", C.c_int64), ("slo_lo", C.c_int64), ("slo_hi", C.c_int64),
+                ("slo_a", C.c_double * MAXN), ("slo_b", C.c_double * MAXN)]
 
 
 class OraSummary(C.Structure):
     _fields_ = [("sum_p", C.c_double), ("sumsq_p", C.c_double), ("max_p", C.c_double),
                 ("sum_theta", C.c_double), ("n_window", C.c_int32), ("n_viol", C.c_int32),
-                ("act_count", C.c_int32 * MAXM)]
+                ("act_count", C.c_int32 * MAXM), ("n_miss", C.c_int32)]
 
 
 class OraModel(C.Structure):
@@ -80,6 +82,9 @@ def lib():
         dp, ip = C.POINTER(C.c_double), C.POINTER(C.c_int32)
         cp = C.POINTER(OraCfg)
         L.ora_levels.argtypes = [cp, C.c_int, dp, dp, dp]
+        L.ora_slo_level.argtypes = [cp, C.c_int, C.c_double, dp]
+        L.ora_slo_bounds.argtypes = [cp, C.POINTER(OraWorkload), C.c_int64, dp, ip]
+        L.ora_slo_bounds.restype = C.c_uint32
         L.ora_identify_ls.argtypes = [C.c_int, C.c_int, dp, dp, dp, dp, dp]
         L.ora_sweep_rows.argtypes = [cp, C.c_uint64, C.c_int, dp, dp]
         L.ora_sweep_nrows.argtypes = [cp]
@@ -157,6 +162,11 @@ def make_workload(desc: dict, periods: int | None = None) -> OraWorkload:
     w.cap_frac0, w.cap_frac_rand, w.cap_frac_step = wl["cap_frac0"], wl["cap_frac_rand"], wl["cap_frac_step"]
     w.cap_period, w.cap_lo, w.cap_hi, w.cap_mult = wl["cap_period"], wl["cap_lo"], wl["cap_hi"], wl["cap_mult"]
     w.gain_dlo, w.gain_step = wl.get("gain_dlo", 0.0), wl.get("gain_step", 0.0)
+    w.slo_period, w.slo_lo, w.slo_hi = wl.get("slo_period", 0), wl.get("slo_lo", 0), wl.get("slo_hi", 0)
+    for j, r in enumerate(wl.get("slo_a") or []):
+        w.slo_a[j] = r
+    for j, r in enumerate(wl.get("slo_b") or []):
+        w.slo_b[j] = r
     return w
 
 
@@ -177,6 +187,19 @@ class Oracle:
         lv, mid, g = np.zeros(L), np.zeros(max(L - 1, 1)), np.zeros(L)
         self.L.ora_levels(C.byref(self.cfg), j, _dp(lv), _dp(mid), _dp(g))
         return lv, mid[: L - 1], g
+
+    # ---- SLO (NEXT-1)
+    def slo_level(self, j, ratio):
+        fr = np.zeros(1)
+        q = self.L.ora_slo_level(C.byref(self.cfg), j, float(ratio), _dp(fr))
+        return int(q), float(fr[0])
+
+    def slo_bounds(self, k, periods=None):
+        w = make_workload(self.desc, periods)
+        lo = np.zeros(self.n); q = np.zeros(self.n, dtype=np.int32)
+        st = self.L.ora_slo_bounds(C.byref(self.cfg), C.byref(w), int(k), _dp(lo),
+                                   q.ctypes.data_as(C.POINTER(C.c_int32)))
+        return lo, q, int(st)
 
     # ---- S0
     def identify_ls(self, F, p):
@@ -382,11 +405,12 @@ def summaries_to_numpy(summ, M):
     ni = len(summ)
     d = dict(sum_p=np.zeros(ni), sumsq_p=np.zeros(ni), max_p=np.zeros(ni), sum_theta=np.zeros(ni),
              n_window=np.zeros(ni, dtype=np.int32), n_viol=np.zeros(ni, dtype=np.int32),
-             act_count=np.zeros((ni, M), dtype=np.int32))
+             act_count=np.zeros((ni, M), dtype=np.int32), n_miss=np.zeros(ni, dtype=np.int32))
     for i, s in enumerate(summ):
         d["sum_p"][i], d["sumsq_p"][i], d["max_p"][i] = s.sum_p, s.sumsq_p, s.max_p
         d["sum_theta"][i], d["n_window"][i], d["n_viol"][i] = s.sum_theta, s.n_window, s.n_viol
         d["act_count"][i] = list(s.act_count)[:M]
+        d["n_miss"][i] = s.n_miss
     return d
 
 
