@@ -161,7 +161,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab"])
+    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo"])
     ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -170,7 +170,10 @@ def parse():
 
 
 def workload_name(d, periods):
-    label = f"cfg{d['cfg']}" if isinstance(d["cfg"], int) else "stability sweep (NEXT-4, gains as caps)"
+    label = f"cfg{d['cfg']}" if isinstance(d["cfg"], int) else {
+        "stability": "stability sweep (NEXT-4, gains as caps)",
+        "slo": "SLO schedule (NEXT-1, §6.4: 50 %-tail SLOs, GPU0 -> 30 % / GPU1-2 -> 80 % tail in [14, 114) mod 200)",
+    }[d["cfg"]]
     return (f"{label}: {d['n_servers']:,} servers x {d['workload']['n_caps']} caps, 1 CPU + "
             f"{d['n_gpus']} GPUs (N={d['n_gpus'] + 1}), P/M={d['P']}/{d['M']}, {periods} periods per step")
 

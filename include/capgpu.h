@@ -116,6 +116,17 @@ typedef struct {
   double gain_dlo, gain_step; /* gain-mismatch sweep (NEXT-4, §4.4): the plant of cap
                                  index c has true gains g_c a with g_c = 1 + gain_dlo + c gain_step
                                  (0, 0 -> the nominal plant) */
+  /* Time-varying latency SLOs (NEXT-1, §6.4; Eq. 10b-c; DESIGN.md
+   * Q29-Q31).  slo_a / slo_b [knob] = SLO_j / e_min,j (0 = no SLO for that knob).
+   * Phase B is in force at instant k while slo_period > 0 and k mod slo_period lies
+   * in [slo_lo, slo_hi); phase A otherwise (slo_period = 0: phase A throughout).
+   * Knob j's lower bound at instant k is max(f_lo_j, level(q_j)), q_j = the lowest
+   * grid level whose latency e_min (f_max/level)^gamma meets the SLO; an SLO no
+   * level meets (ratio < 1) pins the bound to f_max and sets CAPGPU_ST_SLO_INFEASIBLE.
+   * A delta-sigma sub-step whose level index is below q_j is a deadline miss
+   * (capgpu_trace.n_miss_d).  Not supported with `hierarchical`. */
+  int64_t slo_period, slo_lo, slo_hi;
+  double slo_a[CAPGPU_MAX_KNOBS], slo_b[CAPGPU_MAX_KNOBS];
 } capgpu_workload;
 
 /* Optional outputs of capgpu_simulate; every pointer may be NULL.
@@ -127,6 +138,7 @@ typedef struct {
   int32_t *n_viol_d, *n_window_d;                      /* [n_inst] */
   int32_t *act_count_d;                                /* [M][n_inst] */
   double *final_p_d;                                   /* [n_inst] p(k0+K) */
+  int32_t *n_miss_d;                                   /* [n_inst] SLO deadline misses (sub-steps x knobs) */
   int32_t n_trace;
   const int64_t *trace_inst_d;                         /* [n_trace] local instance ids */
   double *p_d, *cap_d;                                 /* [K][n_trace] p(k), P_s(k) */

@@ -54,7 +54,9 @@ class Workload(C.Structure):
                 ("cap_lo", C.c_int64), ("cap_hi", C.c_int64), ("cap_mult", C.c_double),
                 ("hierarchical", C.c_int32), ("rack", C.c_int32), ("block", C.c_int32),
                 ("cluster_frac", C.c_double), ("rack_frac", C.c_double), ("cap_base_d", _VP),
-                ("gain_dlo", C.c_double), ("gain_step", C.c_double)]
+                ("gain_dlo", C.c_double), ("gain_step", C.c_double),
+                ("slo_period", C.c_int64), ("slo_lo", C.c_int64), ("slo_hi", C.c_int64),
+                ("slo_a", C.c_double * MAX_KNOBS), ("slo_b", C.c_double * MAX_KNOBS)]
 
 
 _VP = C.c_void_p
@@ -62,7 +64,7 @@ _VP = C.c_void_p
 
 class Trace(C.Structure):
     _fields_ = [("sum_p_d", _VP), ("sumsq_p_d", _VP), ("max_p_d", _VP), ("sum_theta_d", _VP),
-                ("n_viol_d", _VP), ("n_window_d", _VP), ("act_count_d", _VP), ("final_p_d", _VP),
+                ("n_viol_d", _VP), ("n_window_d", _VP), ("act_count_d", _VP), ("final_p_d", _VP), ("n_miss_d", _VP),
                 ("n_trace", C.c_int32), ("trace_inst_d", _VP), ("p_d", _VP), ("cap_d", _VP), ("u_d", _VP),
                 ("ahat_d", _VP), ("theta_d", _VP), ("active_d", _VP), ("rank_d", _VP), ("levels_d", _VP),
                 ("status_d", _VP), ("agg_W_d", _VP), ("agg_P_d", _VP)]
@@ -205,6 +207,11 @@ def workload_from(desc: dict) -> Workload:
     w.rack, w.block = wl.get("rack", 16), wl.get("block", 1024)
     w.cluster_frac, w.rack_frac = wl.get("cluster_frac", 0.55), wl.get("rack_frac", 0.9)
     w.gain_dlo, w.gain_step = wl.get("gain_dlo", 0.0), wl.get("gain_step", 0.0)
+    w.slo_period, w.slo_lo, w.slo_hi = wl.get("slo_period", 0), wl.get("slo_lo", 0), wl.get("slo_hi", 0)
+    for j, r in enumerate(wl.get("slo_a") or []):
+        w.slo_a[j] = r
+    for j, r in enumerate(wl.get("slo_b") or []):
+        w.slo_b[j] = r
     return w
 
 
@@ -309,7 +316,8 @@ class CapGPU:
         ni, M = self.n_inst, self.M
         e = lambda *s, dtype=torch.float64: torch.empty(*s, dtype=dtype, device=self.device)  # noqa: E731
         return dict(sum_p=e(ni), sumsq_p=e(ni), max_p=e(ni), sum_theta=e(ni), n_viol=e(ni, dtype=torch.int32),
-                    n_window=e(ni, dtype=torch.int32), act_count=e(M, ni, dtype=torch.int32), final_p=e(ni))
+                    n_window=e(ni, dtype=torch.int32), act_count=e(M, ni, dtype=torch.int32), final_p=e(ni),
+                    n_miss=e(ni, dtype=torch.int32))
 
     def simulate(self, periods: int, workload: Workload, trace_inst=None, summaries: bool = True,
                  traces=("p", "cap", "u", "ahat", "theta", "active", "rank", "levels", "status"), out=None):
@@ -324,7 +332,8 @@ class CapGPU:
         if out is None:
             out = self.summary_buffers() if summaries else {}
         if summaries:
-            for k in ("sum_p", "sumsq_p", "max_p", "sum_theta", "n_viol", "n_window", "act_count", "final_p"):
+            for k in ("sum_p", "sumsq_p", "max_p", "sum_theta", "n_viol", "n_window", "act_count", "final_p",
+                      "n_miss"):
                 setattr(tr, k + "_d", _ptr(out[k]).value)
         if trace_inst is not None:
             ti = torch.as_tensor(trace_inst, dtype=torch.int64, device=self.device)

@@ -28,6 +28,8 @@ struct capgpu_ctx {
   void *ws = nullptr;
   int64_t ws_bytes = 0;
   bool servers_ready = false, has_prior = false, sim_ready = false;
+  int32_t convex_static = 1;       // dp.convex of the static bounds (control_step, SLO-free runs)
+  KnobConst *kdev_slo = nullptr;   // device [2][CAPGPU_MAX_KNOBS]: knob constants of the SLO phases
   int64_t k_global = 0;
   capgpu_workload wl{};
   Budget budget{};
@@ -277,6 +279,8 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   }
   d.convex = 1;
   for (int j = 0; j < N; ++j) d.convex &= d.k[j].lo == d.k[j].m ? 1 : 0;
+  c->convex_static = d.convex;
+  d.slo = 0;
 
   // ---- state workspace (SoA)
   const int64_t ni = c->n_inst, ns = c->n_srv;
@@ -284,7 +288,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   const int64_t nd_srv = (int64_t)(5 * N + 3);
   const int64_t grid_bytes = (int64_t)sizeof(GridEntry) * n_class * CAPGPU_MAX_LEVELS;
   const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 12 * (int64_t)h.M * ni + 4 * ni + grid_bytes +
-                        (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 256;
+                        (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS * 3 + 256;
   cudaError_t e = cudaMalloc(&c->ws, (size_t)bytes);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -320,6 +324,9 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   KnobConst *kdev = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 7) / 8);
   cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice);
   d.k_dev = kdev;
+  c->kdev_slo = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS * 2 + 7) / 8);
+  d.k_dev_slo[0] = c->kdev_slo;
+  d.k_dev_slo[1] = c->kdev_slo + CAPGPU_MAX_KNOBS;
   s.trace_slot = (int32_t *)q;
   s.act = (uint32_t *)(s.trace_slot + ni);
   for (int c2 = 0; c2 < n_class; ++c2)
@@ -436,7 +443,10 @@ int capgpu_control_step(capgpu_ctx *c, const double *p_meas_d, const double *f_a
   OPT_DEV(c, ahat_out_d);
   OPT_DEV(c, status_out_d);
   if (!c->has_prior) return fail(c, CAPGPU_E_ORDER, "no prior A0: call capgpu_identify or capgpu_set_prior first");
-  int e = c->L.control_step(c->dp, c->st, p_meas_d, f_applied_d, thr_d, thr_max_d, cap_d, u_out_d, active_out_d,
+  DevParams dp = c->dp;  // static bounds: no SLO schedule on user measurements
+  dp.slo = 0;
+  dp.convex = c->convex_static;
+  int e = c->L.control_step(dp, c->st, p_meas_d, f_applied_d, thr_d, thr_max_d, cap_d, u_out_d, active_out_d,
                             rank_out_d, ahat_out_d, status_out_d, (cudaStream_t)stream);
   if (e) return cuda_fail(c, (cudaError_t)e, "control_step");
   return CAPGPU_OK;
@@ -460,6 +470,68 @@ int capgpu_sim_reset(capgpu_ctx *c) {
   c->sim_ready = false;
   c->budget.ready = false;
   c->k_global = 0;
+  return CAPGPU_OK;
+}
+
+// NEXT-1: the SLO schedule's per-phase bounds (§6.4, Eq. 10b-c
+// P:205-208; Q29-Q31).  Host-side constants only (like the grid table): for
+// each phase and knob the SLO level q = the lowest grid level whose latency
+// e_min (f_max/level)^gamma meets SLO = ratio e_min, i.e. level >= f_max
+// ratio^(-1/gamma); bound = max(f_lo, level(q)), or f_max + SLO_INFEASIBLE when
+// no level meets it.  Validation happens before anything is launched.
+static int apply_slo(capgpu_ctx *c, const capgpu_workload &w, cudaStream_t s) {
+  DevParams &d = c->dp;
+  d.slo = 0;
+  d.convex = c->convex_static;
+  bool any = false;
+  for (int j = 0; j < CAPGPU_MAX_KNOBS; ++j) {
+    if (!(w.slo_a[j] >= 0.0) || !(w.slo_b[j] >= 0.0) || !std::isfinite(w.slo_a[j]) || !std::isfinite(w.slo_b[j]))
+      return fail(c, CAPGPU_E_INVALID, "slo ratios must be finite and >= 0");
+    if (j >= c->N && (w.slo_a[j] != 0.0 || w.slo_b[j] != 0.0))
+      return fail(c, CAPGPU_E_INVALID, "slo ratio set for knob %d >= N", j);
+    any |= w.slo_a[j] != 0.0 || w.slo_b[j] != 0.0;
+  }
+  if (!any) return CAPGPU_OK;
+  if (w.hierarchical) return fail(c, CAPGPU_E_UNSUPPORTED, "SLO schedule with the hierarchical budget");
+  if (w.slo_period < 0 || (w.slo_period > 0 && !(w.slo_lo >= 0 && w.slo_lo <= w.slo_hi)))
+    return fail(c, CAPGPU_E_INVALID, "slo schedule");
+  KnobConst kk[2][CAPGPU_MAX_KNOBS];
+  int convex = 1;
+  for (int ph = 0; ph < 2; ++ph) {
+    uint32_t st = 0u;
+    for (int j = 0; j < CAPGPU_MAX_KNOBS; ++j) {
+      kk[ph][j] = d.k[j];
+      d.q_slo[ph][j] = 0;
+      if (j >= c->N) continue;
+      const double ratio = ph ? w.slo_b[j] : w.slo_a[j];
+      if (ratio > 0.0) {
+        const capgpu_knob_bounds &b = c->bounds[j];
+        const double step = (b.f_max - b.f_min) / (double)(b.n_levels - 1);
+        const double f_req = b.f_max * std::pow(ratio, -1.0 / c->prm.gamma);
+        int q = b.n_levels;
+        double lev = b.f_max;
+        for (int l = 0; l < b.n_levels; ++l) {
+          const double lv = b.f_min + (double)l * step;
+          if (lv >= f_req) {
+            q = l;
+            lev = lv;
+            break;
+          }
+        }
+        if (q >= b.n_levels) st |= CAPGPU_ST_SLO_INFEASIBLE;
+        kk[ph][j].lo = q >= b.n_levels ? b.f_max : (lev > d.k[j].lo ? lev : d.k[j].lo);
+        d.q_slo[ph][j] = q;
+      }
+      convex &= kk[ph][j].lo == kk[ph][j].m ? 1 : 0;
+    }
+    d.st_slo[ph] = st;
+  }
+  CK_CUDA(c, cudaMemcpyAsync(c->kdev_slo, kk, sizeof kk, cudaMemcpyHostToDevice, s));
+  d.slo = 1;
+  d.slo_period = w.slo_period;
+  d.slo_lo = w.slo_lo;
+  d.slo_hi = w.slo_hi;
+  d.convex = convex;
   return CAPGPU_OK;
 }
 
@@ -526,6 +598,7 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
     t.n_viol = tr->n_viol_d;
     t.n_window = tr->n_window_d;
     t.act_count = tr->act_count_d;
+    t.n_miss = tr->n_miss_d;
     t.n_trace = tr->n_trace;
     t.p = tr->p_d;
     t.cap = tr->cap_d;
@@ -538,6 +611,11 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
     t.levels = tr->levels_d;
   }
   if (wl->cap_base_d) NEED_DEV(c, wl->cap_base_d);
+  OPT_DEV(c, tr ? tr->n_miss_d : nullptr);
+  {
+    int rc = apply_slo(c, *wl, s);
+    if (rc) return rc;
+  }
   apply_workload(c->dp, *wl);
   if (!c->sim_ready) {
     int rc = ensure_servers(c, s);

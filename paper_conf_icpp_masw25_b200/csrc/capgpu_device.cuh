@@ -78,6 +78,15 @@ struct DevParams {
   int64_t n_srv, n_inst;     // local counts
   const GridEntry *grid;     // device [n_class][kMaxL]
   const KnobConst *k_dev;    // device copy of k[] for out-of-line code (keeps P in the param bank)
+  // SLO schedule (NEXT-1, §6.4, Eq. 10b-c; Q29-Q31).  Phase B at instant k
+  // while slo_period > 0 and k mod slo_period in [slo_lo, slo_hi).  k_dev_slo[ph]
+  // = device copy of k[] with phase ph's lower bounds; q_slo[ph][j] = SLO level
+  // index (0 = no SLO, L = unreachable); st_slo[ph] = SLO_INFEASIBLE or 0.
+  int32_t slo;               // 1 iff an SLO is in force in either phase
+  int64_t slo_period, slo_lo, slo_hi;
+  const KnobConst *k_dev_slo[2];
+  int32_t q_slo[2][kMaxN];
+  uint32_t st_slo[2];
   long long *phase;          // [8][n_inst] cycle counters (builds with -DCAPGPU_PHASE_TIMING only)
   KnobConst k[kMaxN];
 };
@@ -548,10 +557,14 @@ __device__ __forceinline__ int level_of(const KnobConst &kc, const GridEntry *ta
   return l + (v > mm.y ? 1 : 0) - (v <= mm.x ? 1 : 0);
 }
 
-template <int N>
+// MISS: also count the SLO deadline misses of the period (Q31): sub-steps whose
+// level index lies below the SLO level q_slo[phase][j] of the instant.
+template <int N, bool MISS = false>
 __device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const GridEntry *grid, const double (&u0)[N],
                                                   double (&acc)[N], const double (&dem)[N],
-                                                  const double (&thr_max)[N], double (&fbar)[N], double (&thr)[N]) {
+                                                  const double (&thr_max)[N], double (&fbar)[N], double (&thr)[N],
+                                                  int phase = 0, int *miss = nullptr) {
+  int nm = 0;
   double fs[N], ts[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
@@ -566,6 +579,7 @@ __device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const Grid
       const GridEntry *tab = grid + kc.cls * kMaxL;
       const double v = __dadd_rn(u0[j], acc[j]);
       const int l = level_of<N>(kc, tab, v);
+      if constexpr (MISS) nm += l < P.q_slo[phase][j] ? 1 : 0;
       const double2 lg = __ldg(reinterpret_cast<const double2 *>(&tab[l].level));
       acc[j] = __dadd_rn(v, -lg.x);
       fs[j] = __dadd_rn(fs[j], lg.x);
@@ -578,6 +592,7 @@ __device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const Grid
     fbar[j] = __dmul_rn(fs[j], P.inv_S);
     thr[j] = __dmul_rn(ts[j], P.inv_S);
   }
+  if constexpr (MISS) *miss += nm;
 }
 
 // The same plant for a compile-time sub-step count S (the fused kernel's
@@ -590,10 +605,12 @@ __device__ __forceinline__ void plant_delta_sigma(const DevParams &P, const Grid
 // the capacities min(dem, thr_max g) are formed once per candidate.  Knobs
 // outer, sub-steps unrolled: the knobs' serial acc chains interleave.  Same
 // arithmetic, same order as plant_delta_sigma (bit-identical results).
-template <int N, int S>
+template <int N, int S, bool MISS = false>
 __device__ __forceinline__ void plant_delta_sigma_c(const DevParams &P, const GridEntry *grid, const double (&u0)[N],
                                                     double (&acc)[N], const double (&dem)[N],
-                                                    const double (&thr_max)[N], double (&fbar)[N], double (&thr)[N]) {
+                                                    const double (&thr_max)[N], double (&fbar)[N], double (&thr)[N],
+                                                    int phase = 0, int *miss = nullptr) {
+  int nm = 0;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     const KnobConst &kc = P.k[j];
@@ -608,6 +625,8 @@ __device__ __forceinline__ void plant_delta_sigma_c(const DevParams &P, const Gr
     const double k0 = __dmul_rn(tm, c0.y), kl = __dmul_rn(tm, cl.y), kh = __dmul_rn(tm, ch.y);
     const double t0 = d < k0 ? d : k0, tl = d < kl ? d : kl, th = d < kh ? d : kh;
     double a = acc[j], fs = 0.0, ts = 0.0;
+    int qj = 0;
+    if constexpr (MISS) qj = P.q_slo[phase][j] - l;  // miss <=> l + up - dn < q  <=>  up - dn < q - l
 #pragma unroll
     for (int s = 0; s < S; ++s) {
       const double v = __dadd_rn(u0[j], a);
@@ -617,11 +636,13 @@ __device__ __forceinline__ void plant_delta_sigma_c(const DevParams &P, const Gr
       a = __dadd_rn(v, -lev);
       fs = __dadd_rn(fs, lev);
       ts = __dadd_rn(ts, tt);
+      if constexpr (MISS) nm += ((int)up - (int)dn) < qj ? 1 : 0;
     }
     acc[j] = a;
     fbar[j] = __dmul_rn(fs, P.inv_S);
     thr[j] = __dmul_rn(ts, P.inv_S);
   }
+  if constexpr (MISS) *miss += nm;
 }
 
 // Trace of the level indices (traced instances only): replays the same

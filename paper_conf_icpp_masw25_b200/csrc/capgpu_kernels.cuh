@@ -35,7 +35,7 @@ struct StatePtrs {
 
 struct TracePtrs {
   double *sum_p, *sumsq_p, *max_p, *sum_theta, *final_p;
-  int32_t *n_viol, *n_window, *act_count;
+  int32_t *n_viol, *n_window, *act_count, *n_miss;
   int32_t n_trace;
   double *p, *cap, *u, *ahat, *theta;
   uint32_t *active, *status;
@@ -315,12 +315,14 @@ struct InstantOut {
 // roots s_t (warm starts for the next period), the per-block active codes and
 // the status; returns mean_j theta_j.  Only short-lived temporaries are kept
 // in registers (the caller's state lives in the slab / registers it owns).
-template <int N, int M, bool SCALED = false, class SAcc, class VAcc, class A0Acc, class TAcc, class TmAcc>
+template <int N, int M, bool SCALED = false, bool SLO = false, class SAcc, class VAcc, class A0Acc, class TAcc,
+          class TmAcc>
 __device__ __forceinline__ double control_instant(const DevParams &P, double inv_lam_k, double cap, double &w, VAcc mu_f,
                                                   double &mu_p, SAcc S, VAcc Sfp, A0Acc A0,
                                                   const double (&fbar)[N], double p, TAcc thr, TmAcc thr_max,
                                                   double (&s_prev)[M], uint32_t (&act)[M], double (&u0)[N],
-                                                  uint32_t &status, const InstantOut &out, int64_t inst = 0) {
+                                                  uint32_t &status, const InstantOut &out, int64_t inst = 0,
+                                                  int phase = 0) {
   (void)inst;
   CAPGPU_PHASE_DECL
   // S1 (Eq. 5; Q1-Q4)
@@ -365,15 +367,17 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
   }
   CAPGPU_MARK(P, 3, inst);
   // S3 (Eq. 9-10a)
-  double beta = p - cap, smin = 0.0, smax = 0.0;
+  double beta = p - cap;
 #pragma unroll
-  for (int j = 0; j < N; ++j) {
-    beta = fma(-ahat[j], fbar[j], beta);
-    smin = fma(ahat[j], P.k[j].lo, smin);
-    smax = fma(ahat[j], P.k[j].hi, smax);
-  }
-  status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
+  for (int j = 0; j < N; ++j) beta = fma(-ahat[j], fbar[j], beta);
   if (P.convex) {
+    double smin = 0.0, smax = 0.0;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      smin = fma(ahat[j], P.k[j].lo, smin);
+      smax = fma(ahat[j], P.k[j].hi, smax);
+    }
+    status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
     // all M blocks in lock-step (independent chains interleave; one code copy)
     double s[M];
     solve_blocks_convex<N, M>(P, ahat, tau, beta + smin, act, s);
@@ -396,30 +400,36 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
     }
     return tsum * P.inv_N;
   }
-  // General (non-convex) path: blocks t = 0..M-1, one loop body (not
-  // unrolled: instruction cache); the per-block registers rotate so the body
-  // indexes no array by t.  act[] holds last period's codes on entry (warm
-  // start) and this period's on exit.
-  double ad[N];
+  // General (non-convex) path: SLO-raised lower bounds (l != m).  The knob
+  // constants come from the device copy of this instant's SLO phase (NEXT-1;
+  // without an SLO schedule the static bounds, k_dev).  Blocks t = 0..M-1, one
+  // loop body (not unrolled: instruction cache); the per-block registers
+  // rotate so the body indexes no array by t.  act[] holds last period's codes
+  // on entry (warm start) and this period's on exit.
+  const KnobConst *kc = SLO ? P.k_dev_slo[phase] : P.k;
+  const KnobConst *kc_dev = SLO ? kc : P.k_dev;
+  {
+    double smin = 0.0, smax = 0.0;
 #pragma unroll
-  for (int j = 0; j < N; ++j) ad[j] = ahat[j] * P.k[j].span;
+    for (int j = 0; j < N; ++j) {
+      smin = fma(ahat[j], kc[j].lo, smin);
+      smax = fma(ahat[j], kc[j].hi, smax);
+    }
+    status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
+    if constexpr (SLO) status |= P.st_slo[phase];
+  }
 #pragma unroll 1
   for (int t = 0; t < M; ++t) {
     double ctau[N];
     const double c = P.ct[t];
 #pragma unroll
     for (int j = 0; j < N; ++j) ctau[j] = c * tau[j];
-    uint32_t code = act[0];
-    double s;
-    if (P.convex) {
-      s = solve_block_convex<N>(P.k, ahat, ad, ctau, beta, smin, code);
-    } else {
-      s = solve_block<N>(P.k, P.k_dev, ahat, ctau, beta, s_prev[0]);
-      code = block_codes<N>(P.k, ctau, s);
-    }
+    uint32_t code;
+    const double s = solve_block<N>(kc, kc_dev, ahat, ctau, beta, s_prev[0]);
+    code = block_codes<N>(kc, ctau, s);
     if (t == 0 || out.u) {
       double u[N];
-      code = block_u<N>(P.k, ctau, s, u);
+      code = block_u<N>(kc, ctau, s, u);
       if (t == 0) {
 #pragma unroll
         for (int j = 0; j < N; ++j) u0[j] = u[j];
@@ -497,7 +507,9 @@ struct SimOccupancy {
 #endif
 };
 
-template <int N, int M, int S, int BLOCK>
+// SLO: the NEXT-1 SLO-schedule instantiation (phase tracking, per-phase bounds,
+// miss counting); SLO-free runs use the SLO = false code, unchanged.
+template <int N, int M, int S, int BLOCK, bool SLO = false>
 __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
     k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
   using SL = SlabLayout<N>;
@@ -567,7 +579,9 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   // ---- summaries (Q25)
   const int kw = K - (4 * K) / 5;
   double sum_p = 0.0, sumsq_p = 0.0, max_p = 0.0, sum_theta = 0.0;
-  int n_viol = 0;
+  int n_viol = 0, n_miss = 0;
+  // SLO schedule position r = k mod slo_period (NEXT-1), advanced per period
+  int64_t slo_r = SLO && P.slo_period > 0 ? k0 % P.slo_period : 0;
   int act_cnt[M];
 #pragma unroll
   for (int t = 0; t < M; ++t) act_cnt[t] = 0;
@@ -596,8 +610,13 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
     }
     CAPGPU_MARK(P, 7, i);
     inv_lam_k *= P.inv_lam;
-    const double tbar = control_instant<N, M, true>(P, inv_lam_k, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
-                                              act, u0, status, io, i);
+    int phase = 0;
+    if constexpr (SLO) {
+      phase = slo_r >= P.slo_lo && slo_r < P.slo_hi ? 1 : 0;
+      if (P.slo_period > 0 && ++slo_r == P.slo_period) slo_r = 0;
+    }
+    const double tbar = control_instant<N, M, true, SLO>(P, inv_lam_k, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
+                                              act, u0, status, io, i, phase);
     CAPGPU_MARK(P, 0, i);
     if (slot >= 0) {
       const int64_t b = (int64_t)kk * tr.n_trace + slot;
@@ -631,10 +650,19 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
       plant_trace_levels<N>(P.k_dev, P.S, sgrid, u_l, a_l, tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot,
                             tr.n_trace);
     }
-    if constexpr (S > 0)
-      plant_delta_sigma_c<N, S>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
-    else
-      plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+    if constexpr (SLO) {  // NEXT-1: the same plant, counting the SLO deadline misses (Q31)
+      int m = 0;
+      if constexpr (S > 0)
+        plant_delta_sigma_c<N, S, true>(P, sgrid, u0, acc, dem, thr_max, fbar, thr, phase, &m);
+      else
+        plant_delta_sigma<N, true>(P, sgrid, u0, acc, dem, thr_max, fbar, thr, phase, &m);
+      if (kk >= kw) n_miss += m;
+    } else {
+      if constexpr (S > 0)
+        plant_delta_sigma_c<N, S>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+      else
+        plant_delta_sigma<N>(P, sgrid, u0, acc, dem, thr_max, fbar, thr);
+    }
     CAPGPU_MARK(P, 5, i);
     const double noise = gen_noise(knoise, k + 1, P.noise_scale);
     double pw = c_true;
@@ -681,6 +709,7 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   if (tr.max_p) tr.max_p[i] = max_p;
   if (tr.sum_theta) tr.sum_theta[i] = sum_theta;
   if (tr.n_viol) tr.n_viol[i] = n_viol;
+  if (tr.n_miss) tr.n_miss[i] = n_miss;
   if (tr.n_window) tr.n_window[i] = K - kw;
   if (tr.final_p) tr.final_p[i] = p;
   if (tr.act_count) {
@@ -836,6 +865,7 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
       if (tr.sum_theta) tr.sum_theta[i] = (first ? 0.0 : tr.sum_theta[i]) + tbar;
       if (tr.n_viol) tr.n_viol[i] = (first ? 0 : tr.n_viol[i]) + (p_next > cap ? 1 : 0);
       if (tr.n_window) tr.n_window[i] = K - kw;
+      if (tr.n_miss && first) tr.n_miss[i] = 0;  // no SLO schedule with the budget
       if (tr.act_count) {
 #pragma unroll
         for (int t = 0; t < M; ++t) tr.act_count[t * ld + i] = (first ? 0 : tr.act_count[t * ld + i]) + (act[t] != 0u);
@@ -1079,11 +1109,11 @@ struct LaunchN {
 // Fused-kernel launch: block size chosen so that the last wave is nearly full
 // (the per-instance period chain is serial, so a ragged last wave costs a
 // whole per-instance run time).
-template <int N, int M, int S, int BLOCK>
+template <int N, int M, int S, int BLOCK, bool SLO = false>
 int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
   const int smem = (int)(sizeof(double) * SlabLayout<N>::F * BLOCK);
-  cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  k_simulate<N, M, S, BLOCK><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
+  cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK, SLO>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  k_simulate<N, M, S, BLOCK, SLO><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
   return (int)cudaGetLastError();
 }
 
@@ -1137,6 +1167,7 @@ struct LaunchNM {
       const double nb = std::ceil((double)P.n_inst / block);
       return std::ceil(nb / sms) * block * (1.0 + 0.02 * (8.0 / (occ * block / 32.0)));
     };
+    if (P.slo) return launch_sim<N, M, S, 32, true>(P, st, tr, k0, K, s);  // NEXT-1 (one block size)
     if (occ128[nc] <= 0 || busiest(occ32[nc], 32) < busiest(occ128[nc], 128))
       return launch_sim<N, M, S, 32>(P, st, tr, k0, K, s);
     return launch_sim<N, M, S, 128>(P, st, tr, k0, K, s);
