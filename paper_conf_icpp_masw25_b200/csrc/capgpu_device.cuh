@@ -120,13 +120,14 @@ __device__ __forceinline__ double plant_gain(const DevParams &P, int cidx) {
 }
 
 __device__ __forceinline__ double rcp_fast(double x) {
-  // MUFU.RCP64H seed + two Newton steps: ~1 ulp (continuous quantities only).
+  // MUFU.RCP64H seed y0 with residual e = 1 - x y0, |e| < 2^-20, then
+  // 1/x = y0 / (1 - e) = y0 (1 + e + e^2) + O(e^3): three dependent FMAs
+  // (two Newton steps need four) for ~1 ulp (continuous quantities only;
+  // tools/dbg/rcp_check.cu measures it on the device).
   double y;
   asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
-  double e = fma(-x, y, 1.0);
-  y = fma(y, e, y);
-  e = fma(-x, y, 1.0);
-  return fma(y, e, y);
+  const double e = fma(-x, y, 1.0);
+  return fma(y, fma(e, e, e), y);
 }
 
 __device__ __forceinline__ long long dbits(double x) { return __double_as_longlong(x); }
@@ -183,17 +184,25 @@ __device__ __forceinline__ void model_push(double lam, double inv_lam_k, double 
 
 // In-register LDL^T solve of a packed SPD system: A (packed upper, destroyed
 // into the factors), b -> x.  Used for the model (S1) and identification (S0).
+//
+// Critical path.  Column j waits for d_j, which waits for dinv_{j-1} through
+// the last term L(j,j-1) W(j,j-1) of its sum, W(i,k) = L(i,k) D_k being the
+// unnormalised column.  W(j,j-1) is kept from column j-1 (wp[]) instead of
+// being re-formed as L(j,j-1) D_{j-1}, so the chain per column is one DMUL
+// (L = W dinv), one DFMA and the 3-deep reciprocal; the other W(j,k) are
+// re-formed off the critical path.
 template <int N>
 __device__ __forceinline__ void ldlt_solve(double (&L)[Tri<N>::size], const double (&b)[N], double (&x)[N]) {
   double dinv[N];
+  double wp[N];  // wp[i] = W(i, j-1) of the previous column (rows i >= j)
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     double v[N > 1 ? N - 1 : 1];
     double d = L[Tri<N>::idx(j, j)];
 #pragma unroll
     for (int k = 0; k < j; ++k) {
-      // v_k = L(j,k) D_k with the unit-lower factor L(j,k) of column k
-      v[k] = L[Tri<N>::idx(j, k)] * L[Tri<N>::idx(k, k)];
+      // v_k = W(j,k) = L(j,k) D_k with the unit-lower factor L(j,k) of column k
+      v[k] = k == j - 1 ? wp[j] : L[Tri<N>::idx(j, k)] * L[Tri<N>::idx(k, k)];
       d = fma(-L[Tri<N>::idx(j, k)], v[k], d);
     }
     L[Tri<N>::idx(j, j)] = d;
@@ -203,6 +212,7 @@ __device__ __forceinline__ void ldlt_solve(double (&L)[Tri<N>::size], const doub
       double y = L[Tri<N>::idx(i, j)];
 #pragma unroll
       for (int k = 0; k < j; ++k) y = fma(-L[Tri<N>::idx(i, k)], v[k], y);
+      wp[i] = y;
       L[Tri<N>::idx(i, j)] = y * dinv[j];
     }
   }
@@ -216,9 +226,10 @@ __device__ __forceinline__ void ldlt_solve(double (&L)[Tri<N>::size], const doub
   }
 #pragma unroll
   for (int i = N - 1; i >= 0; --i) {
+    // x_{i+1} (the most recent) enters last: a linear, not quadratic, chain
     double t = y[i] * dinv[i];
 #pragma unroll
-    for (int k = i + 1; k < N; ++k) t = fma(-L[Tri<N>::idx(k, i)], x[k], t);
+    for (int k = N - 1; k > i; --k) t = fma(-L[Tri<N>::idx(k, i)], x[k], t);
     x[i] = t;
   }
 }
@@ -364,139 +375,56 @@ __device__ __noinline__ double block_exact(const KnobConst *kc, const double *a_
   return num * rcp_fast(den);
 }
 
-// Convex case (no SLO-raised lower bound: lo_j == m_j for all j).  For s >= 0
-// every knob sits at lo (phi(s) = s - beta - a.lo); for s < 0 every knob is
-// free or at its upper bound, u_j(s) = min(m_j - c tau_j s, hi_j), and phi is
-// convex.  Hence:
-//   beta + a.lo >= 0  ->  s* = beta + a.lo exactly (all knobs at lo);
-//   otherwise the piece with upper set U has the root
-//     s_U = (beta + a.lo + sum_{j in U} a_j (hi_j - m_j)) / (1 + sum_{j not in U} c tau_j a_j)
-//   and, phi being convex, every piece line lies below phi, so s_U >= s*.
-//   Starting from last period's U, s_U >= s* and U(s_U) is a subset of U(s*);
-//   iterating U <- U(s_U) moves s down monotonically and stops exactly when
-//   the set reproduces itself: the exact root, in at most N + 1 steps.
-// No phi evaluation is needed: one piece root and one classification per step.
-// code: in = previous period's codes of this block, out = codes at the root.
+// One convex block (weight c), exact: iterate U <- U(s_U) from the start set
+// `up` (upper bits 2j+1).  Any start set works: every piece line of the convex
+// phi lies below phi, so s_U >= s* and U(s_U) is a subset of U(s*); s moves
+// down monotonically and stops on the root's piece (<= N + 1 steps).  The set
+// sums are predicated adds (no 0/1 masks); the classification is Q19's
+// v_j = m_j - c tau_j s > h_j written as -(c s) tau_j > h_j - m_j.
+//   ta_j = tau_j a_j, ad_j = a_j (h_j - m_j), TA = sum_j ta_j, base = beta + a.l < 0.
 template <int N>
-__device__ __forceinline__ double solve_block_convex(const KnobConst *kc, const double (&a)[N],
-                                                     const double (&ad)[N], const double (&ctau)[N],
-                                                     double beta, double a_lo_sum, uint32_t &code) {
-  const double base = beta + a_lo_sum;
-  if (!(base < 0.0)) {
-    uint32_t c = 0u;
-#pragma unroll
-    for (int j = 0; j < N; ++j) c |= (base > 0.0 && ctau[j] > 0.0 ? 1u : 0u) << (2 * j);
-    code = c;
-    return base;
-  }
-  double cta[N], den_all = 1.0;
-#pragma unroll
-  for (int j = 0; j < N; ++j) {
-    cta[j] = ctau[j] * a[j];
-    den_all += cta[j];
-  }
-  uint32_t up = code & 0xAAAAAAAAu;  // previous upper set (bit 2j+1)
+__device__ __forceinline__ double convex_root(const KnobConst *kc, double c, const double (&tau)[N],
+                                              const double (&ta)[N], const double (&ad)[N], double base, double TA,
+                                              uint32_t &up) {
   double s = 0.0;
 #pragma unroll 1
   for (int it = 0; it <= N; ++it) {
-    // branch-free: 0/1 mask per knob (one FSEL), two partial sums each for ILP
-    double num0 = base, num1 = 0.0, den0 = den_all, den1 = 0.0;
+    double n0 = base, n1 = 0.0, d0 = 0.0, d1 = 0.0;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
-      const double mk = ((up >> (2 * j + 1)) & 1u) ? 1.0 : 0.0;
-      if (j & 1) {
-        num1 = fma(mk, ad[j], num1);
-        den1 = fma(-mk, cta[j], den1);
-      } else {
-        num0 = fma(mk, ad[j], num0);
-        den0 = fma(-mk, cta[j], den0);
+      if ((up >> (2 * j + 1)) & 1u) {
+        if (j & 1) {
+          n1 += ad[j];
+          d1 += ta[j];
+        } else {
+          n0 += ad[j];
+          d0 += ta[j];
+        }
       }
     }
-    s = (num0 + num1) * rcp_fast(den0 + den1);
+    s = (n0 + n1) * rcp_fast(fma(c, TA - (d0 + d1), 1.0));
+    const double mcs = -c * s;
     uint32_t nu = 0u;
 #pragma unroll
-    for (int j = 0; j < N; ++j) nu |= (fma(-ctau[j], s, kc[j].m) > kc[j].hi ? 2u : 0u) << (2 * j);
+    for (int j = 0; j < N; ++j) nu |= (mcs * tau[j] > kc[j].span ? 2u : 0u) << (2 * j);
     if (nu == up) break;
     up = nu;
   }
-  code = up;
   return s;
 }
 
-// All M blocks of the convex case at once (same structure as
-// solve_block_convex).  Shared across blocks: base = beta + a.lo (the
-// all-low test does not depend on c_t), ta_j = tau_j a_j with TA = sum ta_j,
-// ad_j = a_j (h_j - m_j), and the upper thresholds b_j = -(h_j - m_j)/tau_j:
-//   knob j is at its upper bound  <=>  m_j - c tau_j s > h_j  <=>  c s < b_j.
-// Per block and step: s_U = (base + sum_U ad_j) / (1 + c (TA - sum_U ta_j)).
-// The blocks iterate in lock-step (independent dependency chains interleave).
-// act: in = last period's codes (warm start), out = upper codes at the roots.
-template <int N, int M>
-__device__ __forceinline__ void solve_blocks_convex(const DevParams &P, const double (&a)[N], const double (&tau)[N],
-                                                    double base, uint32_t (&act)[M], double (&s)[M]) {
-  if (!(base < 0.0)) {  // root s* = base >= 0 in every block: all knobs at lo
-    uint32_t c = 0u;
+// Does the convex block with weight c have any bound active at its root?
+// U(s*) is empty iff U(s_0) is, s_0 = base / (1 + c TA) being the all-free
+// root (U only grows as s decreases, and s* <= s_0).  The fused kernel needs
+// only this bit for the blocks it does not apply or trace (act_count summary).
+template <int N>
+__device__ __forceinline__ bool convex_any_upper(const KnobConst *kc, double c, const double (&tau)[N], double base,
+                                                 double TA) {
+  const double mcs = -c * (base * rcp_fast(fma(c, TA, 1.0)));
+  bool any = false;
 #pragma unroll
-    for (int j = 0; j < N; ++j) c |= (base > 0.0 && tau[j] > 0.0 ? 1u : 0u) << (2 * j);
-#pragma unroll
-    for (int t = 0; t < M; ++t) {
-      s[t] = base;
-      act[t] = c;
-    }
-    return;
-  }
-  double ta[N], ad[N], b[N], TA0 = 0.0, TA1 = 0.0;
-#pragma unroll
-  for (int j = 0; j < N; ++j) {
-    ta[j] = tau[j] * a[j];
-    ad[j] = a[j] * P.k[j].span;
-    b[j] = -P.k[j].span * rcp_fast(tau[j]);  // tau_j = 0 -> -inf: never upper
-    if (j & 1) TA1 += ta[j]; else TA0 += ta[j];
-  }
-  const double TA = TA0 + TA1;
-  uint32_t up[M];
-  bool done[M];
-#pragma unroll
-  for (int t = 0; t < M; ++t) {
-    up[t] = act[t] & 0xAAAAAAAAu;
-    done[t] = false;
-    s[t] = 0.0;
-  }
-#pragma unroll 1
-  for (int it = 0; it <= N; ++it) {
-    bool all = true;
-#pragma unroll
-    for (int t = 0; t < M; ++t) {
-      if (done[t]) continue;
-      double n0 = base, n1 = 0.0, d0 = 0.0, d1 = 0.0;
-#pragma unroll
-      for (int j = 0; j < N; ++j) {
-        const double mk = ((up[t] >> (2 * j + 1)) & 1u) ? 1.0 : 0.0;
-        if (j & 1) {
-          n1 = fma(mk, ad[j], n1);
-          d1 = fma(mk, ta[j], d1);
-        } else {
-          n0 = fma(mk, ad[j], n0);
-          d0 = fma(mk, ta[j], d0);
-        }
-      }
-      const double c = P.ct[t];
-      const double st = (n0 + n1) * rcp_fast(fma(c, TA - (d0 + d1), 1.0));
-      const double cs = c * st;
-      uint32_t nu = 0u;
-#pragma unroll
-      for (int j = 0; j < N; ++j) nu |= (cs < b[j] ? 2u : 0u) << (2 * j);
-      s[t] = st;
-      if (nu == up[t]) done[t] = true;
-      else {
-        up[t] = nu;
-        all = false;
-      }
-    }
-    if (all) break;
-  }
-#pragma unroll
-  for (int t = 0; t < M; ++t) act[t] = up[t];
+  for (int j = 0; j < N; ++j) any |= mcs * tau[j] > kc[j].span;
+  return any;
 }
 
 // Solve one block; returns the root s (u and codes follow from it).

@@ -309,6 +309,8 @@ struct InstantOut {
   double *u, *ahat, *theta;  // [M][N], [N], [N]
   int8_t *rank;              // [N]
   int64_t ld;
+  bool full;                 // exact codes of every block wanted (traces, control_step); else blocks
+                             // 1..M-1 report only whether a bound is active (summaries)
 };
 
 // One control instant for one instance: S1, S2, S3.  Leaves u0 (block 0), the
@@ -378,9 +380,49 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
       smax = fma(ahat[j], P.k[j].hi, smax);
     }
     status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
-    // all M blocks in lock-step (independent chains interleave; one code copy)
+    // Blocks 0..M-2 share the weight c = Q (Q11), so they are ONE problem;
+    // block M-1 (c = (P-M+1) Q) is solved exactly only when its codes are
+    // wanted (out.full), else only its "any bound active" bit is formed.
+    const double base = beta + smin;
     double s[M];
-    solve_blocks_convex<N, M>(P, ahat, tau, beta + smin, act, s);
+    if (!(base < 0.0)) {  // root s* = base >= 0 in every block: all knobs at lo
+      uint32_t c = 0u;
+#pragma unroll
+      for (int j = 0; j < N; ++j) c |= (base > 0.0 && tau[j] > 0.0 ? 1u : 0u) << (2 * j);
+#pragma unroll
+      for (int t = 0; t < M; ++t) {
+        s[t] = base;
+        act[t] = c;
+      }
+    } else {
+      double ta[N], ad[N], TA0 = 0.0, TA1 = 0.0;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        ta[j] = tau[j] * ahat[j];
+        ad[j] = ahat[j] * P.k[j].span;
+        if (j & 1) TA1 += ta[j]; else TA0 += ta[j];
+      }
+      const double TA = TA0 + TA1;
+      const bool any_last = M > 1 && !out.full ? convex_any_upper<N>(P.k, P.ct[M - 1], tau, base, TA) : false;
+      uint32_t up0 = act[0] & 0xAAAAAAAAu;
+      const double s0 = convex_root<N>(P.k, P.ct[0], tau, ta, ad, base, TA, up0);
+#pragma unroll
+      for (int t = 0; t + 1 < M; ++t) {
+        s[t] = s0;
+        act[t] = up0;
+      }
+      if (M == 1) {
+        s[0] = s0;
+        act[0] = up0;
+      } else if (out.full) {
+        uint32_t upl = act[M - 1] & 0xAAAAAAAAu;
+        s[M - 1] = convex_root<N>(P.k, P.ct[M - 1], tau, ta, ad, base, TA, upl);
+        act[M - 1] = upl;
+      } else {
+        s[M - 1] = s0;  // warm start only (never used by the convex path)
+        act[M - 1] = any_last ? 2u : 0u;
+      }
+    }
 #pragma unroll
     for (int t = 0; t < M; ++t) s_prev[t] = s[t];
     double ctau[N];
@@ -603,6 +645,7 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
     InstantOut io{};
     if (slot >= 0) {
       io.ld = tr.n_trace;
+      io.full = true;
       io.u = tr.u ? tr.u + (int64_t)kk * M * N * tr.n_trace + slot : nullptr;
       io.ahat = tr.ahat ? tr.ahat + (int64_t)kk * N * tr.n_trace + slot : nullptr;
       io.theta = tr.theta ? tr.theta + (int64_t)kk * N * tr.n_trace + slot : nullptr;
@@ -814,6 +857,7 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
     InstantOut io{};
     if (slot >= 0) {
       io.ld = tr.n_trace;
+      io.full = true;
       io.u = tr.u ? tr.u + (int64_t)kk * M * N * tr.n_trace + slot : nullptr;
       io.ahat = tr.ahat ? tr.ahat + (int64_t)kk * N * tr.n_trace + slot : nullptr;
       io.theta = tr.theta ? tr.theta + (int64_t)kk * N * tr.n_trace + slot : nullptr;
@@ -982,7 +1026,7 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
   }
   const GlobAcc S{st.S + i, ld};
   double u0[N];
-  InstantOut io{u_out + i, ahat_out ? ahat_out + i : nullptr, nullptr, rank_out ? rank_out + i : nullptr, ld};
+  InstantOut io{u_out + i, ahat_out ? ahat_out + i : nullptr, nullptr, rank_out ? rank_out + i : nullptr, ld, true};
   control_instant<N, M>(P, 0.0, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
                         RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
   st.w[i] = w;
