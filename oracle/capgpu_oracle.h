@@ -63,6 +63,12 @@ typedef struct {
    * otherwise. */
   int64_t slo_period, slo_lo, slo_hi;
   double slo_a[ORA_MAXN], slo_b[ORA_MAXN];
+  /* Baseline controllers (NEXT-2, §6.1; Q32-Q35) replacing S1-S3:
+   * 0 = CapGPU (MPC), 1 = Fixed-step, 2 = Safe Fixed-step, 3 = GPU-only, 4 = CPU-only. */
+  int32_t controller;
+  int32_t fs_levels;   /* Fixed-step size in grid levels (stepsize 1 or 5) */
+  double safe_margin;  /* Safe Fixed-step: set point lowered by this many W */
+  double p_pole;       /* GPU-/CPU-only: closed-loop pole z of the pole-placed P gain */
 } ora_workload;
 
 /* per-instance summary over the last 80 % of periods */
@@ -147,6 +153,13 @@ int ora_simulate(const ora_cfg *c, const ora_workload *w, int n_inst, const int6
                  uint8_t *tr_levels /*[S][N]*/, double *tr_ahat /*[N]*/, double *tr_theta /*[N]*/,
                  uint32_t *tr_status, double *final_p /*[n_inst]: p(K)*/, ora_summary *summ,
                  double *A0_out /*[n_inst][N]*/, int use_definition_mode);
+
+/* ---- baseline controllers (NEXT-2): same plant, S1-S3 replaced by the
+ * controller of w->controller (Q32-Q35).  Traces as ora_simulate: tr_u holds
+ * the command [N] (row 0 only), tr_theta the weights the controller saw. */
+int ora_simulate_baseline(const ora_cfg *c, const ora_workload *w, int n_inst, const int64_t *inst,
+                          double *tr_p, double *tr_cap, double *tr_u /*[N]*/, uint8_t *tr_levels /*[S][N]*/,
+                          double *tr_theta /*[N]*/, double *final_p, ora_summary *summ);
 
 /* ---- S5 hierarchical budget (cfg 4, Q16) */
 int ora_simulate_hier(const ora_cfg *c, const ora_workload *w, int n_servers, int rack, double cluster_frac,

@@ -57,7 +57,9 @@ class OraWorkload(C.Structure):
                 ("cap_period", C.c_int64), ("cap_lo", C.c_int64), ("cap_hi", C.c_int64),
                 ("cap_mult", C.c_double), ("gain_dlo", C.c_double), ("gain_step", C.c_double),
                 ("slo_period", C.c_int64), ("slo_lo", C.c_int64), ("slo_hi", C.c_int64),
-                ("slo_a", C.c_double * MAXN), ("slo_b", C.c_double * MAXN)]
+                ("slo_a", C.c_double * MAXN), ("slo_b", C.c_double * MAXN),
+                ("controller", C.c_int32), ("fs_levels", C.c_int32), ("safe_margin", C.c_double),
+                ("p_pole", C.c_double)]
 
 
 class OraSummary(C.Structure):
@@ -117,6 +119,8 @@ def lib():
                                    dp, C.POINTER(OraSummary), dp, C.c_int]
         L.ora_budget_caps.argtypes = [C.c_int, C.c_int, dp, dp, C.c_double, C.c_double,
                                       C.c_double, dp, dp]
+        L.ora_simulate_baseline.argtypes = [cp, wp, C.c_int, C.POINTER(C.c_int64), dp, dp, dp,
+                                            C.POINTER(C.c_uint8), dp, dp, C.POINTER(OraSummary)]
         L.ora_simulate_hier.argtypes = [cp, wp, C.c_int, C.c_int, C.c_double, C.c_double, dp, C.c_double,
                                         C.c_int, C.c_int, C.POINTER(C.c_int64), dp, dp, dp, u32p, u32p,
                                         C.POINTER(C.c_uint8), dp, dp, dp]
@@ -167,6 +171,8 @@ def make_workload(desc: dict, periods: int | None = None) -> OraWorkload:
         w.slo_a[j] = r
     for j, r in enumerate(wl.get("slo_b") or []):
         w.slo_b[j] = r
+    w.controller, w.fs_levels = wl.get("controller", 0), wl.get("fs_levels", 1)
+    w.safe_margin, w.p_pole = wl.get("safe_margin", 0.0), wl.get("p_pole", 0.5)
     return w
 
 
@@ -363,6 +369,31 @@ class Oracle:
         out["final_p"] = final_p
         out["A0"] = A0
         out["summary"] = summaries_to_numpy(summ, M)
+        return out
+
+    def simulate_baseline(self, inst, periods=None, traces=True):
+        """NEXT-2 baseline controller of the workload (controller 1..4) on the same plant."""
+        inst = np.ascontiguousarray(np.asarray(inst, dtype=np.int64))
+        ni = len(inst)
+        w = make_workload(self.desc, periods)
+        K, n, S = w.periods, self.n, self.S
+        out = {}
+        if traces:
+            out = dict(p=np.zeros((K, ni)), cap=np.zeros((K, ni)), u=np.zeros((K, ni, n)),
+                       levels=np.zeros((K, ni, S, n), dtype=np.uint8), theta=np.zeros((K, ni, n)))
+        final_p = np.zeros(ni)
+        summ = (OraSummary * ni)()
+
+        def P(name, ct=C.c_double):
+            return out[name].ctypes.data_as(C.POINTER(ct)) if traces else None
+
+        rc = self.L.ora_simulate_baseline(C.byref(self.cfg), C.byref(w), ni, inst.ctypes.data_as(C.POINTER(C.c_int64)),
+                                          P("p"), P("cap"), P("u"), P("levels", C.c_uint8), P("theta"),
+                                          _dp(final_p), summ)
+        if rc != 0:
+            raise RuntimeError(f"ora_simulate_baseline rc={rc}")
+        out["final_p"] = final_p
+        out["summary"] = summaries_to_numpy(summ, self.M)
         return out
 
     def simulate_hier(self, n_servers, tr_srv, periods=None, W_replay=None, W0_replay=0.0, n_total=None):
