@@ -425,10 +425,21 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
     }
 #pragma unroll
     for (int t = 0; t < M; ++t) s_prev[t] = s[t];
-    double ctau[N];
+    // u of block 0 at its root.  base >= 0: every knob at l (codes as above);
+    // else s < 0, so v_j = m_j - c tau_j s >= m_j = l_j: a knob is free or upper.
+    {
+      const double mcs = -P.ct[0] * s[0];
+      uint32_t code = 0u;
 #pragma unroll
-    for (int j = 0; j < N; ++j) ctau[j] = P.ct[0] * tau[j];
-    act[0] = block_u<N>(P.k, ctau, s[0], u0);
+      for (int j = 0; j < N; ++j) {
+        const double v = fma(mcs, tau[j], P.k[j].m);
+        const bool up = v > P.k[j].hi;
+        code |= (up ? 2u : 0u) << (2 * j);
+        u0[j] = base < 0.0 ? (up ? P.k[j].hi : v) : P.k[j].lo;
+      }
+      if (base < 0.0) act[0] = code;
+    }
+    double ctau[N];
     if (out.u) {
 #pragma unroll 1
       for (int t = 0; t < M; ++t) {
