@@ -161,7 +161,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo"])
+    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo", "fixed", "safe", "gpuonly", "cpuonly"])
     ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -173,7 +173,7 @@ def workload_name(d, periods):
     label = f"cfg{d['cfg']}" if isinstance(d["cfg"], int) else {
         "stability": "stability sweep (NEXT-4, gains as caps)",
         "slo": "SLO schedule (NEXT-1, §6.4: 50 %-tail SLOs, GPU0 -> 30 % / GPU1-2 -> 80 % tail in [14, 114) mod 200)",
-    }[d["cfg"]]
+    }.get(d["cfg"], f"NEXT-2 baseline controller {d['cfg'][9:]} on the cfg 2 plant")
     return (f"{label}: {d['n_servers']:,} servers x {d['workload']['n_caps']} caps, 1 CPU + "
             f"{d['n_gpus']} GPUs (N={d['n_gpus'] + 1}), P/M={d['P']}/{d['M']}, {periods} periods per step")
 
@@ -316,7 +316,9 @@ def main():
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_value = total_per_step * len(e2e_evs) / float(te.item())
 
-    flops = algorithmic_flops(N, M, S)
+    ctrl = d["workload"].get("controller", 0)
+    # NEXT-2 baselines: the plant (S4) + the S2 weights + the rule; no S1 / S3
+    flops = algorithmic_flops(N, M, S) if ctrl == 0 else (4 * N * S + 7 * N + 6) + 4 * N + 4
     launch_s = t_local / args.steps
     if hier:
         # per-period mode: the state streams through HBM every period
@@ -353,7 +355,8 @@ def main():
                                    "(DESIGN.md §8); measured DFMA microbench in peak_measured",
                     "peak_measured": measured_peak,
                     "state_bytes_per_step": state_bytes_per_instance(N, M) / periods}
-            mode = "fused multi-period kernel k_simulate (1 launch per step)"
+            mode = ("fused multi-period kernel k_simulate (1 launch per step)" if ctrl == 0 else
+                    "fused multi-period baseline kernel k_baseline (1 launch per step)")
             par = f"dp{world} (server shards, no data-path collective)"
             launches = args.steps
         line = {"metric": "server-control-steps/sec", "value": value, "unit": "server-control-steps/s",

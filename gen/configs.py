@@ -117,11 +117,15 @@ def baseline(controller: str, n_servers: int = 1024, periods: int = 1000, fs_lev
 def by_name(name) -> dict:
     """bench.py --config: "1".."5" (BASELINE.json configs), "stab" (the NEXT-4
     gain sweep at bench size: 16,384 servers x 24 gains x 1,000 periods) or
-    "slo" (the NEXT-1 SLO schedule: 1,048,576 servers x 1,000 periods)."""
+    "slo" (the NEXT-1 SLO schedule: 1,048,576 servers x 1,000 periods), or a
+    NEXT-2 baseline "fixed" / "safe" / "gpuonly" / "cpuonly" (1,048,576 servers
+    of the cfg 2 plant x 1,000 periods)."""
     if str(name) == "stab":
         return stability_sweep(n_servers=16384)
     if str(name) == "slo":
         return slo_schedule(n_servers=1048576)
+    if str(name) in CONTROLLERS and str(name) != "capgpu":
+        return baseline(str(name), n_servers=1048576)
     return get(int(name))
 
 

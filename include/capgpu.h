@@ -127,7 +127,23 @@ typedef struct {
    * (capgpu_trace.n_miss_d).  Not supported with `hierarchical`. */
   int64_t slo_period, slo_lo, slo_hi;
   double slo_a[CAPGPU_MAX_KNOBS], slo_b[CAPGPU_MAX_KNOBS];
+  /* Controller (NEXT-2, §6.1; Q32-Q35): CAPGPU_CTRL_*.  The
+   * baselines replace S1-S3 on the same plant: Fixed-step moves the movable knob
+   * with the highest (p < P_s) or lowest (p > P_s) theta by fs_levels grid levels
+   * (ties round-robin; Safe Fixed-step uses P_s - safe_margin); GPU-only / CPU-only
+   * run g(k) = clamp(g(k-1) + K (P_s - p(k))) on one common GPU (CPU) frequency
+   * with the other knobs at f_max and the pole-placed gain K = (1 - p_pole) / sum_J A0_j.
+   * Traces: u row 0 = the command, theta, p, cap, levels; status 0; act_count 0.
+   * The controller is fixed for a simulation (first call after create/sim_reset).
+   * Not supported with `hierarchical`. */
+  int32_t controller;
+  int32_t fs_levels;   /* >= 1 */
+  double safe_margin;  /* W, finite */
+  double p_pole;       /* in [0, 1) */
 } capgpu_workload;
+
+enum { CAPGPU_CTRL_CAPGPU = 0, CAPGPU_CTRL_FIXED_STEP = 1, CAPGPU_CTRL_SAFE_FIXED_STEP = 2,
+       CAPGPU_CTRL_GPU_ONLY = 3, CAPGPU_CTRL_CPU_ONLY = 4 };
 
 /* Optional outputs of capgpu_simulate; every pointer may be NULL.
  * Summaries are over the last floor(0.8 K) of the K periods of the call (Q25).

@@ -547,6 +547,10 @@ static void apply_workload(DevParams &d, const capgpu_workload &w) {
   d.cap_mult = w.cap_mult;
   d.gain0 = 1.0 + w.gain_dlo;
   d.gain_step = w.gain_step;
+  d.bl_kind = w.controller;
+  d.bl_steps = w.fs_levels;
+  d.bl_margin = w.safe_margin;
+  d.bl_pole = w.p_pole;
 }
 
 }  // extern "C"
@@ -566,6 +570,15 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
     return fail(c, CAPGPU_E_INVALID, "gain_dlo / gain_step must be finite");
   if (wl->hierarchical && (wl->gain_dlo != 0.0 || wl->gain_step != 0.0))
     return fail(c, CAPGPU_E_INVALID, "gain mismatch is not supported with the hierarchical budget");
+  if (wl->controller < CAPGPU_CTRL_CAPGPU || wl->controller > CAPGPU_CTRL_CPU_ONLY)
+    return fail(c, CAPGPU_E_INVALID, "controller");
+  if (wl->controller != CAPGPU_CTRL_CAPGPU) {
+    if (wl->hierarchical) return fail(c, CAPGPU_E_UNSUPPORTED, "baseline controllers with the hierarchical budget");
+    if (wl->fs_levels < 1 || !std::isfinite(wl->safe_margin) || !(wl->p_pole >= 0.0 && wl->p_pole < 1.0))
+      return fail(c, CAPGPU_E_INVALID, "baseline parameters (fs_levels >= 1, finite safe_margin, 0 <= p_pole < 1)");
+  }
+  if (c->sim_ready && wl->controller != c->wl.controller)
+    return fail(c, CAPGPU_E_ORDER, "the controller is fixed for a simulation: call capgpu_sim_reset first");
   if (tr) {
     OPT_DEV(c, tr->sum_p_d);
     OPT_DEV(c, tr->sumsq_p_d);
@@ -691,6 +704,9 @@ int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, c
     rc = budget_simulate(c->budget, c->dp, c->st, t, c->L, c->k_global, periods, tr ? tr->agg_W_d : nullptr,
                          tr ? tr->agg_P_d : nullptr, s, c->err);
     if (rc) return rc;
+  } else if (wl->controller != CAPGPU_CTRL_CAPGPU) {
+    int e = c->L.baseline(c->dp, c->st, t, c->k_global, (int)periods, s);
+    if (e) return cuda_fail(c, (cudaError_t)e, "simulate (baseline controller)");
   } else {
     int e = c->L.simulate(c->dp, c->st, t, c->k_global, (int)periods, s);
     if (e) return cuda_fail(c, (cudaError_t)e, "simulate");

@@ -87,6 +87,10 @@ struct DevParams {
   const KnobConst *k_dev_slo[2];
   int32_t q_slo[2][kMaxN];
   uint32_t st_slo[2];
+  // Baseline controllers (NEXT-2, §6.1; Q32-Q35): 0 = CapGPU MPC,
+  // 1 = Fixed-step, 2 = Safe Fixed-step, 3 = GPU-only, 4 = CPU-only.
+  int32_t bl_kind, bl_steps;
+  double bl_margin, bl_pole;
   long long *phase;          // [8][n_inst] cycle counters (builds with -DCAPGPU_PHASE_TIMING only)
   KnobConst k[kMaxN];
 };

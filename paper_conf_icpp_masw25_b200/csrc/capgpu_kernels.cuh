@@ -772,6 +772,207 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
   }
 }
 
+// Dynamic index into a small register array without local memory: an
+// unrolled compare/select chain.
+template <int N>
+__device__ __forceinline__ int st_lev_get(const int (&a)[N], int j) {
+  int r = a[0];
+#pragma unroll
+  for (int q = 1; q < N; ++q) r = j == q ? a[q] : r;
+  return r;
+}
+template <int N>
+__device__ __forceinline__ void st_lev_set(int (&a)[N], int j, int v) {
+#pragma unroll
+  for (int q = 0; q < N; ++q) a[q] = j == q ? v : a[q];
+}
+template <int N>
+__device__ __forceinline__ double reg_get(const double (&a)[N], int j) {
+  double r = a[0];
+#pragma unroll
+  for (int q = 1; q < N; ++q) r = j == q ? a[q] : r;
+  return r;
+}
+
+// ------------------------------------------------------------------ baseline controllers (NEXT-2)
+//
+// The paper's comparison controllers (§6.1) on the same plant:
+// S1-S3 are replaced by
+//   Fixed-step (Q32): all knobs start at their lowest
+//     level; if p < P_s (Safe: P_s - margin) the movable knob with
+//     the highest normalised utilisation theta moves up `bl_steps` levels, if
+//     p > P_s the movable knob with the lowest moves down; ties go round-robin
+//     (first tied knob at or after pointer rr, then rr = chosen + 1);
+//   GPU-only / CPU-only (Q34-Q35): g(k) = clamp(g(k-1) + K (P_s - p(k)))
+//     on one common GPU (CPU) frequency, the other knobs at f_max, with the
+//     pole-placed gain K = (1 - z) / sum_J A0_j.
+// theta is the IEEE S2 weight (the Fixed-step choice is an integer decision:
+// bit-exact with the oracle).  One thread per instance, state in registers;
+// the baseline state reuses the (unused) model-state arrays: level indices in
+// mu_f, the loop command g in w, the round-robin pointer in act[0].
+template <int N, int S, bool SLO>
+__global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= P.n_inst) return;
+  const int64_t si = i / P.n_caps, ls = P.n_srv, li = P.n_inst;
+  const uint64_t srv = (uint64_t)(P.srv_begin + si);
+  const double gain = plant_gain(P, (int)(i - si * P.n_caps));
+  double fbar[N], acc[N], thr[N], thr_max[N], base[N], amp[N], a_true[N];
+  int lev[N];
+  double sumA = 0.0, g_lo = 0.0, g_hi = 0.0;
+  const int kind = P.bl_kind;
+  const int j0 = kind == 3 ? 1 : 0, j1 = kind == 3 ? N : 1;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    fbar[j] = st.fbar[j * li + i];
+    acc[j] = st.acc[j * li + i];
+    thr[j] = st.thr[j * li + i];
+    lev[j] = (int)st.mu_f[j * li + i];
+    thr_max[j] = st.thr_max[j * ls + si];
+    base[j] = st.base[j * ls + si];
+    amp[j] = st.amp[j * ls + si];
+    a_true[j] = __dmul_rn(gain, st.a_true[j * ls + si]);
+    if (j >= j0 && j < j1) {
+      sumA = __dadd_rn(sumA, st.A0[j * ls + si]);
+      if (j == j0 || P.k[j].f_min < g_lo) g_lo = P.k[j].f_min;
+      if (j == j0 || P.k[j].f_max > g_hi) g_hi = P.k[j].f_max;
+    }
+  }
+  const double Kp = __ddiv_rn(1.0 - P.bl_pole, sumA);
+  double g = st.w[i];
+  if (!(g > 0.0)) g = g_lo;  // first period: the loop starts from the lowest frequency
+  int rr = (int)st.act[i];
+  double p = st.p[i];
+  const double c_true = st.c_true[si], cap_base = st.cap_base[i];
+  const int slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
+  const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
+  const uint64_t kburst = gen_stream_key(P.seed, GEN_TAG_BURST, srv);
+  const uint64_t knoise = gen_stream_key(P.seed, GEN_TAG_NOISE, srv);
+  int64_t epoch = (k0 + 1) / GEN_BURST_HOLD;
+  int left = (int)(GEN_BURST_HOLD - (k0 + 1) % GEN_BURST_HOLD);
+  uint32_t bmask = burst_mask<N>(P, kburst, epoch);
+  const int kw = K - (4 * K) / 5;
+  double sum_p = 0.0, sumsq_p = 0.0, max_p = 0.0, sum_theta = 0.0;
+  int n_viol = 0, n_miss = 0;
+  int64_t slo_r = SLO && P.slo_period > 0 ? k0 % P.slo_period : 0;
+#pragma unroll 1
+  for (int kk = 0; kk < K; ++kk) {
+    const int64_t k = k0 + kk;
+    const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
+    double theta[N], tsum = 0.0;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      theta[j] = pclamp(__ddiv_rn(thr[j], thr_max[j]), P.theta_min, 1.0);
+      tsum += theta[j];
+    }
+    double u0[N];
+    if (kind <= 2) {
+      const double err = (kind == 2 ? __dadd_rn(cap, -P.bl_margin) : cap) - p;
+      if (err != 0.0) {
+        int best = -1;
+        double tb = 0.0;
+#pragma unroll 1
+        for (int q = 0; q < N; ++q) {
+          int j = rr + q;
+          j = j >= N ? j - N : j;
+          const int lj = st_lev_get(lev, j);
+          const bool movable = err > 0.0 ? lj < P.k[j].L - 1 : lj > 0;
+          const double tj = reg_get(theta, j);
+          if (movable && (best < 0 || (err > 0.0 ? tj > tb : tj < tb))) {
+            best = j;
+            tb = tj;
+          }
+        }
+        if (best >= 0) {
+          const int lb = st_lev_get(lev, best);
+          const int nl = err > 0.0 ? min(lb + P.bl_steps, P.k[best].L - 1) : max(lb - P.bl_steps, 0);
+          st_lev_set(lev, best, nl);
+          rr = best + 1 == N ? 0 : best + 1;
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < N; ++j) u0[j] = P.grid[P.k[j].cls * kMaxL + lev[j]].level;
+    } else {
+      g = fmin(fmax(__dadd_rn(g, __dmul_rn(Kp, cap - p)), g_lo), g_hi);
+#pragma unroll
+      for (int j = 0; j < N; ++j)
+        u0[j] = (j >= j0 && j < j1) ? fmin(fmax(g, P.k[j].f_min), P.k[j].f_max) : P.k[j].f_max;
+    }
+    int phase = 0;
+    if constexpr (SLO) {
+      phase = slo_r >= P.slo_lo && slo_r < P.slo_hi ? 1 : 0;
+      if (P.slo_period > 0 && ++slo_r == P.slo_period) slo_r = 0;
+    }
+    if (slot >= 0) {
+      const int64_t b = (int64_t)kk * tr.n_trace + slot;
+      if (tr.p) tr.p[b] = p;
+      if (tr.cap) tr.cap[b] = cap;
+      if (tr.status) tr.status[b] = 0u;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        if (tr.u) tr.u[((int64_t)kk * P.M * N + j) * tr.n_trace + slot] = u0[j];
+        if (tr.theta) tr.theta[((int64_t)kk * N + j) * tr.n_trace + slot] = theta[j];
+      }
+      if (tr.levels) {
+        double u_l[N], a_l[N];
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+          u_l[j] = u0[j];
+          a_l[j] = acc[j];
+        }
+        plant_trace_levels<N>(P.k_dev, P.S, P.grid, u_l, a_l, tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot,
+                              tr.n_trace);
+      }
+    }
+    // ---- S4: period k -> k+1
+    if (left == 0) {
+      ++epoch;
+      left = GEN_BURST_HOLD;
+      bmask = burst_mask<N>(P, kburst, epoch);
+    }
+    --left;
+    double dem[N];
+    demand_all<N>(P, kjit, k + 1, bmask, thr_max, RegArr<N>{base}, RegArr<N>{amp}, dem);
+    int m = 0;
+    if constexpr (S > 0)
+      plant_delta_sigma_c<N, S, SLO>(P, P.grid, u0, acc, dem, thr_max, fbar, thr, phase, &m);
+    else
+      plant_delta_sigma<N, SLO>(P, P.grid, u0, acc, dem, thr_max, fbar, thr, phase, &m);
+    double pw = c_true;
+#pragma unroll
+    for (int j = 0; j < N; ++j) pw = fma(a_true[j], fbar[j], pw);
+    p = pw + gen_noise(knoise, k + 1, P.noise_scale);
+    if (kk >= kw) {
+      sum_theta += tsum * P.inv_N;
+      sum_p += p;
+      sumsq_p = fma(p, p, sumsq_p);
+      max_p = kk == kw ? p : fmax(max_p, p);
+      n_viol += p > cap;
+      n_miss += m;
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    st.fbar[j * li + i] = fbar[j];
+    st.acc[j * li + i] = acc[j];
+    st.thr[j * li + i] = thr[j];
+    st.mu_f[j * li + i] = (double)lev[j];
+  }
+  st.p[i] = p;
+  st.w[i] = g;
+  st.act[i] = (uint32_t)rr;
+  if (tr.sum_p) tr.sum_p[i] = sum_p;
+  if (tr.sumsq_p) tr.sumsq_p[i] = sumsq_p;
+  if (tr.max_p) tr.max_p[i] = max_p;
+  if (tr.sum_theta) tr.sum_theta[i] = sum_theta;
+  if (tr.n_viol) tr.n_viol[i] = n_viol;
+  if (tr.n_miss) tr.n_miss[i] = n_miss;
+  if (tr.n_window) tr.n_window[i] = K - kw;
+  if (tr.final_p) tr.final_p[i] = p;
+  if (tr.act_count)
+    for (int t = 0; t < P.M; ++t) tr.act_count[t * li + i] = 0;
+}
+
 // ------------------------------------------------------------------ hierarchical budget (S5, cfg 4)
 //
 // Q16: racks of `rack` consecutive servers (aligned lane groups of a warp),
@@ -1125,6 +1326,7 @@ struct Launchers {
   int (*period)(const DevParams &, const StatePtrs &, const BudgetDev &, const TracePtrs &, int64_t, int, int,
                 cudaStream_t);
   int (*budget_init)(const DevParams &, const StatePtrs &, const BudgetDev &, double *, cudaStream_t);
+  int (*baseline)(const DevParams &, const StatePtrs &, const TracePtrs &, int64_t, int, cudaStream_t);
 };
 
 inline int grid_for(int64_t n, int block) { return (int)((n + block - 1) / block); }
@@ -1153,6 +1355,17 @@ struct LaunchN {
                        double *dem, double *noise, cudaStream_t s) {
     k_debug_gen<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, k, a, tm, c, dem, noise);
     return (int)cudaGetLastError();
+  }
+  template <int S, bool SLO>
+  static int baseline_s(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K,
+                        cudaStream_t s) {
+    k_baseline<N, S, SLO><<<grid_for(P.n_inst, 128), 128, 0, s>>>(P, st, tr, k0, K);
+    return (int)cudaGetLastError();
+  }
+  static int baseline(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K,
+                      cudaStream_t s) {
+    if (P.S == 4) return P.slo ? baseline_s<4, true>(P, st, tr, k0, K, s) : baseline_s<4, false>(P, st, tr, k0, K, s);
+    return P.slo ? baseline_s<0, true>(P, st, tr, k0, K, s) : baseline_s<0, false>(P, st, tr, k0, K, s);
   }
   static int budget_init(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, double *part_c,
                          cudaStream_t s) {
@@ -1255,6 +1468,7 @@ Launchers make_launchers(int M) {
   L.assign_weights = &LaunchN<N>::assign_weights;
   L.debug_gen = &LaunchN<N>::debug_gen;
   L.budget_init = &LaunchN<N>::budget_init;
+  L.baseline = &LaunchN<N>::baseline;
 #define CAPGPU_SET_M(MM)                                 \
   case MM:                                               \
     L.simulate = &LaunchNM<N, MM>::simulate;             \
