@@ -46,6 +46,7 @@ typedef struct {
   double gamma;      /* latency exponent */
   double noise_std;  /* meter noise sigma (W) */
   uint64_t seed;
+  double wmove;      /* NEXT-3 move suppression weight W (W^2/MHz^2, Q36); 0 = the literal Eq. 9 */
 } ora_cfg;
 
 typedef struct {
@@ -124,6 +125,15 @@ int ora_mpc_stacked(const ora_cfg *c, const double *Ahat, const double *R, doubl
                     uint32_t *active, uint32_t *tie, int *iters);
 int ora_mpc_bruteforce(const ora_cfg *c, const double *Ahat, const double *R, double beta,
                        const double *lo, const double *hi, const double *m, double *u);
+/* NEXT-3 (Q36): Eq. 9 + sum_{t<M} wmove |d(k+t|k)|^2 with u_{-1} = fbar = f(k);
+ * dense generic active set / brute force / literal cost. */
+int ora_mpc_move(const ora_cfg *c, const double *Ahat, const double *R, double beta, const double *fbar,
+                 const double *lo, const double *hi, const double *m, double *u, uint32_t *active, uint32_t *tie,
+                 int *iters);
+int ora_mpc_move_bruteforce(const ora_cfg *c, const double *Ahat, const double *R, double beta, const double *fbar,
+                            const double *lo, const double *hi, const double *m, double *u);
+double ora_mpc_move_cost(const ora_cfg *c, const double *Ahat, const double *R, double beta, const double *fbar,
+                         const double *m, const double *u);
 double ora_mpc_cost(const ora_cfg *c, const double *Ahat, const double *R, double beta,
                     const double *m, const double *u);
 void ora_mpc_classify(const ora_cfg *c, const double *Ahat, const double *R, double beta,

@@ -47,7 +47,7 @@ class OraCfg(C.Structure):
                 ("q", C.c_double), ("theta_min", C.c_double), ("lam", C.c_double),
                 ("rho", C.c_double), ("a_lo", C.c_double), ("a_hi", C.c_double),
                 ("a_floor", C.c_double), ("gamma", C.c_double), ("noise_std", C.c_double),
-                ("seed", C.c_uint64)]
+                ("seed", C.c_uint64), ("wmove", C.c_double)]
 
 
 class OraWorkload(C.Structure):
@@ -100,6 +100,10 @@ def lib():
         u32p = C.POINTER(C.c_uint32)
         L.ora_mpc_stacked.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp, dp, u32p, u32p, ip]
         L.ora_mpc_bruteforce.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp, dp]
+        L.ora_mpc_move.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp, dp, dp, u32p, u32p, ip]
+        L.ora_mpc_move_bruteforce.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp, dp, dp]
+        L.ora_mpc_move_cost.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp]
+        L.ora_mpc_move_cost.restype = C.c_double
         L.ora_mpc_cost.argtypes = [cp, dp, dp, C.c_double, dp, dp]
         L.ora_mpc_cost.restype = C.c_double
         L.ora_mpc_classify.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp, dp, u32p, u32p]
@@ -154,6 +158,7 @@ def make_cfg(desc: dict) -> OraCfg:
     c.a_lo, c.a_hi, c.a_floor = ctl["a_lo"], ctl["a_hi"], ctl["a_floor"]
     c.gamma, c.noise_std = ctl["gamma"], ctl["noise_std"]
     c.seed = desc["seed"]
+    c.wmove = ctl.get("wmove", 0.0)
     return c
 
 
@@ -275,6 +280,30 @@ class Oracle:
                                     tie.ctypes.data_as(C.POINTER(C.c_uint32)),
                                     it.ctypes.data_as(C.POINTER(C.c_int32)))
         return u, act, tie, int(st), int(it[0])
+
+    def mpc_move(self, Ahat, R, beta, fbar, lo, hi, m):
+        """NEXT-3: Eq. 9 + move suppression (cfg wmove), dense generic active set."""
+        Ahat, R, fbar, lo, hi, m = map(_arr, (Ahat, R, fbar, lo, hi, m))
+        u = np.zeros((self.M, self.n))
+        act = np.zeros(self.M, dtype=np.uint32); tie = np.zeros(self.M, dtype=np.uint32)
+        it = np.zeros(1, dtype=np.int32)
+        st = self.L.ora_mpc_move(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(fbar), _dp(lo), _dp(hi),
+                                 _dp(m), _dp(u), act.ctypes.data_as(C.POINTER(C.c_uint32)),
+                                 tie.ctypes.data_as(C.POINTER(C.c_uint32)), it.ctypes.data_as(C.POINTER(C.c_int32)))
+        return u, act, tie, int(st), int(it[0])
+
+    def mpc_move_bruteforce(self, Ahat, R, beta, fbar, lo, hi, m):
+        Ahat, R, fbar, lo, hi, m = map(_arr, (Ahat, R, fbar, lo, hi, m))
+        u = np.zeros((self.M, self.n))
+        rc = self.L.ora_mpc_move_bruteforce(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(fbar), _dp(lo),
+                                            _dp(hi), _dp(m), _dp(u))
+        if rc != 0:
+            raise ValueError("bruteforce needs M*N <= 10")
+        return u
+
+    def mpc_move_cost(self, Ahat, R, beta, fbar, m, u):
+        Ahat, R, fbar, m, u = map(_arr, (Ahat, R, fbar, m, u))
+        return self.L.ora_mpc_move_cost(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(fbar), _dp(m), _dp(u))
 
     def mpc_bruteforce(self, Ahat, R, beta, lo, hi, m):
         Ahat, R, lo, hi, m = map(_arr, (Ahat, R, lo, hi, m))
