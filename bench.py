@@ -161,7 +161,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo", "fixed", "safe", "gpuonly", "cpuonly"])
+    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo", "fixed", "safe", "gpuonly", "cpuonly", "move"])
     ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -173,6 +173,7 @@ def workload_name(d, periods):
     label = f"cfg{d['cfg']}" if isinstance(d["cfg"], int) else {
         "stability": "stability sweep (NEXT-4, gains as caps)",
         "slo": "SLO schedule (NEXT-1, §6.4: 50 %-tail SLOs, GPU0 -> 30 % / GPU1-2 -> 80 % tail in [14, 114) mod 200)",
+        "move": "horizon-active MPC (NEXT-3: Eq. 9 + move suppression, coupled blocks, generic active set)",
     }.get(d["cfg"], f"NEXT-2 baseline controller {d['cfg'][9:]} on the cfg 2 plant")
     return (f"{label}: {d['n_servers']:,} servers x {d['workload']['n_caps']} caps, 1 CPU + "
             f"{d['n_gpus']} GPUs (N={d['n_gpus'] + 1}), P/M={d['P']}/{d['M']}, {periods} periods per step")
@@ -319,6 +320,9 @@ def main():
     ctrl = d["workload"].get("controller", 0)
     # NEXT-2 baselines: the plant (S4) + the S2 weights + the rule; no S1 / S3
     flops = algorithmic_flops(N, M, S) if ctrl == 0 else (4 * N * S + 7 * N + 6) + 4 * N + 4
+    if ctrl == 0 and d["controller"].get("wmove", 0.0) > 0:
+        V = N * M  # NEXT-3: at least one dense (MN)-variable equality-constrained solve per step
+        flops += V ** 3 / 3 + 4 * V * V
     launch_s = t_local / args.steps
     if hier:
         # per-period mode: the state streams through HBM every period

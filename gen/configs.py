@@ -17,7 +17,7 @@ GPU_KNOB = dict(f_min=435.0, f_max=1350.0, n_levels=11, sweep_base=0)   # base =
 
 # Controller constants (Q1, Q4, Q6, Q8, Q21; P = 8 / M = 2 from P:264; gamma P:190)
 CONTROLLER = dict(q=1.0, r0=1e-4, theta_min=0.05, lam=0.95, rho=100.0, a_lo=0.25, a_hi=4.0,
-                  a_floor=1e-3, gamma=0.91, noise_std=11.0, substeps=4)
+                  a_floor=1e-3, gamma=0.91, noise_std=11.0, substeps=4, wmove=0.0)
 
 _BASE_WORKLOAD = dict(n_caps=1, demand_kind=1, demand_frac=0.7, cap_frac0=0.5, cap_frac_rand=0.0,
                       cap_frac_step=0.0, cap_period=0, cap_lo=0, cap_hi=0, cap_mult=1.0,
@@ -114,6 +114,19 @@ def baseline(controller: str, n_servers: int = 1024, periods: int = 1000, fs_lev
     return d
 
 
+def move_suppression(n_servers: int = 64, periods: int = 1000, wmove: float = 2e-4, n_gpus: int = 3,
+                     P: int = 8, M: int = 2) -> dict:
+    """NEXT-3: the horizon-active MPC (Q36) on the paper's 1 CPU + 3 GPU
+    server (P/M = 8/2): Eq. 9 plus wmove |d(k+t|k)|^2 per control step,
+    set points P_min + (0.3 + 0.5 U) dP, bursty demand.  wmove = 2e-4 W^2/MHz^2
+    is twice the base frequency penalty r0 (Q6)."""
+    d = get(5, n_servers=n_servers, periods=periods, wmove=wmove, n_gpus=n_gpus, P=P, M=M)
+    d["knobs"] = knobs(n_gpus)
+    d["workload"].update(n_caps=1, cap_frac0=0.3, cap_frac_rand=0.5, cap_frac_step=0.0)
+    d["cfg"] = "move"
+    return d
+
+
 def by_name(name) -> dict:
     """bench.py --config: "1".."5" (BASELINE.json configs), "stab" (the NEXT-4
     gain sweep at bench size: 16,384 servers x 24 gains x 1,000 periods) or
@@ -124,6 +137,8 @@ def by_name(name) -> dict:
         return stability_sweep(n_servers=16384)
     if str(name) == "slo":
         return slo_schedule(n_servers=1048576)
+    if str(name) == "move":
+        return move_suppression(n_servers=1048576)
     if str(name) in CONTROLLERS and str(name) != "capgpu":
         return baseline(str(name), n_servers=1048576)
     return get(int(name))

@@ -88,6 +88,10 @@ typedef struct {
   int32_t substeps;   /* delta-sigma sub-steps per period S in {1,2,4,8} (Q22) */
   int32_t caps_per_server; /* simulated instances per server (cfg 5: 32), >= 1 */
   uint64_t seed;      /* synthetic-input seed */
+  double wmove;       /* NEXT-3 move suppression (Q36): Eq. 9 + sum_{t<M} wmove |d(k+t|k)|^2,
+                         >= 0 (W^2/MHz^2); 0 = the literal Eq. 9.  > 0 couples the M blocks: solved by a
+                         generic per-instance active set, CUDA path for M * N <= 10, capgpu_simulate only
+                         (not control_step / hierarchical / SLO schedule: CAPGPU_E_UNSUPPORTED) */
 } capgpu_params;
 
 /* Contiguous server range of this process (one process per GPU, §8(e)). */

@@ -40,7 +40,7 @@ class Params(C.Structure):
     _fields_ = [("q", C.c_double), ("r0", C.c_double), ("theta_min", C.c_double), ("lam", C.c_double),
                 ("rho", C.c_double), ("a_lo", C.c_double), ("a_hi", C.c_double), ("a_floor", C.c_double),
                 ("gamma", C.c_double), ("noise_std", C.c_double), ("substeps", C.c_int32),
-                ("caps_per_server", C.c_int32), ("seed", C.c_uint64)]
+                ("caps_per_server", C.c_int32), ("seed", C.c_uint64), ("wmove", C.c_double)]
 
 
 class Shard(C.Structure):
@@ -88,8 +88,9 @@ def lib():
     if _lib is not None:
         return _lib
     path = LIB_PATH
-    if os.environ.get("CAPGPU_LIB_VARIANT") == "timing":  # profiling build (tools/phase_timing.py)
-        path = os.path.join(_PKG, "libcapgpu_timing.so")
+    var = os.environ.get("CAPGPU_LIB_VARIANT")
+    if var:  # experiment / profiling builds (build.py VARIANTS), e.g. "timing" for tools/phase_timing.py
+        path = os.path.join(_PKG, f"libcapgpu_{var}.so")
     if not os.path.exists(path):
         raise RuntimeError(f"{path} missing: run `python -m paper_conf_icpp_masw25_b200.build` "
                            "(there is no CPU fallback)")
@@ -242,6 +243,7 @@ class CapGPU:
         p.rho, p.a_lo, p.a_hi, p.a_floor = controller["rho"], controller["a_lo"], controller["a_hi"], controller["a_floor"]
         p.gamma, p.noise_std, p.substeps = controller["gamma"], controller["noise_std"], controller["substeps"]
         p.caps_per_server, p.seed = caps_per_server, seed
+        p.wmove = controller.get("wmove", 0.0)
         sh = Shard()
         sh.rank, sh.world, sh.srv_begin = rank, world, srv_begin
         sh.n_servers_global = n_servers_global if n_servers_global is not None else srv_begin + n_servers

@@ -168,6 +168,9 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     return fail(nullptr, CAPGPU_E_INVALID, "params out of range");
   if (!(prm.substeps == 1 || prm.substeps == 2 || prm.substeps == 4 || prm.substeps == 8))
     return fail(nullptr, CAPGPU_E_INVALID, "substeps must be 1, 2, 4 or 8");
+  if (!(prm.wmove >= 0.0) || !std::isfinite(prm.wmove)) return fail(nullptr, CAPGPU_E_INVALID, "wmove must be >= 0");
+  if (prm.wmove > 0.0 && h.M * N > kMoveMaxVars)
+    return fail(nullptr, CAPGPU_E_UNSUPPORTED, "move suppression needs M * N <= %d on the CUDA path", kMoveMaxVars);
   for (int j = 0; j < N; ++j) {
     const capgpu_knob_bounds &b = bounds[j];
     if (!(b.f_min < b.f_max) || !std::isfinite(b.f_min) || !std::isfinite(b.f_max))
@@ -221,6 +224,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   d.noise_scale = prm.noise_std * std::sqrt(3.0);
   d.inv_S = 1.0 / (double)prm.substeps;
   d.inv_lam = 1.0 / prm.lambda;
+  d.wmove = prm.wmove;
   // Q11: c_t = Q for t < M-1, c_{M-1} = (P - M + 1) Q
   for (int t = 0; t < h.M; ++t) d.ct[t] = t < h.M - 1 ? prm.q : (double)(h.P - h.M + 1) * prm.q;
   d.seed = prm.seed;
@@ -443,6 +447,7 @@ int capgpu_control_step(capgpu_ctx *c, const double *p_meas_d, const double *f_a
   OPT_DEV(c, ahat_out_d);
   OPT_DEV(c, status_out_d);
   if (!c->has_prior) return fail(c, CAPGPU_E_ORDER, "no prior A0: call capgpu_identify or capgpu_set_prior first");
+  if (c->prm.wmove > 0.0) return fail(c, CAPGPU_E_UNSUPPORTED, "move suppression (wmove > 0) in control_step");
   DevParams dp = c->dp;  // static bounds: no SLO schedule on user measurements
   dp.slo = 0;
   dp.convex = c->convex_static;
@@ -493,6 +498,8 @@ static int apply_slo(capgpu_ctx *c, const capgpu_workload &w, cudaStream_t s) {
   }
   if (!any) return CAPGPU_OK;
   if (w.hierarchical) return fail(c, CAPGPU_E_UNSUPPORTED, "SLO schedule with the hierarchical budget");
+  if (c->prm.wmove > 0.0 && w.controller == CAPGPU_CTRL_CAPGPU)
+    return fail(c, CAPGPU_E_UNSUPPORTED, "SLO schedule with move suppression");
   if (w.slo_period < 0 || (w.slo_period > 0 && !(w.slo_lo >= 0 && w.slo_lo <= w.slo_hi)))
     return fail(c, CAPGPU_E_INVALID, "slo schedule");
   KnobConst kk[2][CAPGPU_MAX_KNOBS];
@@ -577,6 +584,8 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
     if (wl->fs_levels < 1 || !std::isfinite(wl->safe_margin) || !(wl->p_pole >= 0.0 && wl->p_pole < 1.0))
       return fail(c, CAPGPU_E_INVALID, "baseline parameters (fs_levels >= 1, finite safe_margin, 0 <= p_pole < 1)");
   }
+  if (c->prm.wmove > 0.0 && wl->hierarchical)
+    return fail(c, CAPGPU_E_UNSUPPORTED, "move suppression with the hierarchical budget");
   if (c->sim_ready && wl->controller != c->wl.controller)
     return fail(c, CAPGPU_E_ORDER, "the controller is fixed for a simulation: call capgpu_sim_reset first");
   if (tr) {

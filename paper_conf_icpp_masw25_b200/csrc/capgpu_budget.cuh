@@ -9,7 +9,7 @@
 namespace capgpu {
 
 constexpr int kBudgetBlock = 1024;  // servers per reduction block (fixed granularity)
-constexpr int kCta = 128;           // servers per CTA of k_period
+constexpr int kCta = kPeriodCta;    // servers per CTA of k_period
 constexpr int kCtasPerBlock = kBudgetBlock / kCta;
 
 struct Budget {

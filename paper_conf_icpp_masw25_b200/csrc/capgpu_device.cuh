@@ -91,6 +91,7 @@ struct DevParams {
   // 1 = Fixed-step, 2 = Safe Fixed-step, 3 = GPU-only, 4 = CPU-only.
   int32_t bl_kind, bl_steps;
   double bl_margin, bl_pole;
+  double wmove;              // NEXT-3 move-suppression weight W (Q36); 0 = the literal Eq. 9
   long long *phase;          // [8][n_inst] cycle counters (builds with -DCAPGPU_PHASE_TIMING only)
   KnobConst k[kMaxN];
 };
@@ -471,6 +472,128 @@ __device__ __forceinline__ uint32_t block_u(const KnobConst *kc, const double (&
     u[j] = low ? kc[j].lo : (up ? kc[j].hi : v);
   }
   return code;
+}
+
+// ------------------------------------------------------------------ S3 with move suppression (NEXT-3)
+// Eq. 9 + sum_{t<M} W |u_t - u_{t-1}|^2, u_{-1} = f(k) (Q36): the M blocks
+// couple through the increments, so the decoupled block solve no longer
+// applies.  Generic primal active set on the stacked MN-variable box QP
+// (Nocedal & Wright Alg. 16.3 for bounds), per thread, warm-started from last
+// period's active set, fixed iteration cap 3 MN + 3 (CAPGPU_ST_SOLVER_CAP).
+// The equality-constrained subproblem of each iteration is one masked LDL^T of
+// the full MN x MN Hessian (fixed variables -> identity rows), so the code is
+// branch-free and fully unrolled.  Half the Hessian (variable a = t N + j):
+//   H(a, a)  = c_t A_j^2 + R_j + W (1 + [t < M-1])
+//   H(a, b)  = c_t A_j A_k  (same t, k != j);  -W (same j, |t - t'| = 1)
+//   g(a)     = c_t beta A_j - R_j m_j - [t = 0] W f_j
+template <int N, int M>
+__device__ __forceinline__ double move_h(const DevParams &P, const double (&a)[N], const double (&R)[N], int x,
+                                         int y) {
+  const int tx = x / N, jx = x - tx * N, ty = y / N, jy = y - ty * N;
+  if (tx == ty) {
+    double h = P.ct[tx] * a[jx] * a[jy];
+    if (jx == jy) h += R[jx] + P.wmove * (tx < M - 1 ? 2.0 : 1.0);
+    return h;
+  }
+  return (jx == jy && (tx - ty == 1 || ty - tx == 1)) ? -P.wmove : 0.0;
+}
+
+template <int N, int M>
+__device__ __forceinline__ uint32_t move_qp(const DevParams &P, const KnobConst *kc, const double (&a)[N],
+                                            const double (&R)[N], double beta, const double (&f)[N],
+                                            uint32_t (&act)[M], double (&x)[M * N]) {
+  constexpr int V = M * N;
+  double g[V];
+  uint32_t lo_m = 0u, up_m = 0u;  // working set: variable a fixed at its lower / upper bound
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const int v = t * N + j;
+      g[v] = P.ct[t] * beta * a[j] - R[j] * kc[j].m - (t == 0 ? P.wmove * f[j] : 0.0);
+      const uint32_t code = (act[t] >> (2 * j)) & 3u;
+      lo_m |= (code == 1u ? 1u : 0u) << v;
+      up_m |= (code == 2u ? 1u : 0u) << v;
+      x[v] = code == 1u ? kc[j].lo : (code == 2u ? kc[j].hi : pclamp(f[j], kc[j].lo, kc[j].hi));
+    }
+  }
+  double gscale = 1.0;
+#pragma unroll
+  for (int v = 0; v < V; ++v) gscale = fmax(gscale, fabs(g[v]));
+  uint32_t status = CAPGPU_ST_SOLVER_CAP;
+#pragma unroll 1
+  for (int it = 0; it < 3 * V + 3; ++it) {
+    const uint32_t fix = lo_m | up_m;
+    // equality-constrained subproblem on the free set (masked LDL^T)
+    double L[Tri<V>::size], rhs[V], xs[V];
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      const bool fu = (fix >> u) & 1u;
+      double r = -g[u];
+#pragma unroll
+      for (int w = 0; w < V; ++w) {
+        const bool fw = (fix >> w) & 1u;
+        const double h = move_h<N, M>(P, a, R, u, w);
+        if (w >= u) L[Tri<V>::idx(u, w)] = (fu || fw) ? (u == w ? 1.0 : 0.0) : h;
+        if (fw) r = fma(-h, x[w], r);
+      }
+      rhs[u] = fu ? x[u] : r;
+    }
+    ldlt_solve<V>(L, rhs, xs);
+    // ratio test along xs - x over the free variables
+    double alpha = 1.0;
+    int blk = -1;
+    bool blk_up = false;
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      if ((fix >> u) & 1u) continue;
+      const int j = u % N;
+      const double d = xs[u] - x[u];
+      if (xs[u] < kc[j].lo && d < 0.0) {
+        const double al = (kc[j].lo - x[u]) / d;
+        if (al < alpha) { alpha = al; blk = u; blk_up = false; }
+      } else if (xs[u] > kc[j].hi && d > 0.0) {
+        const double al = (kc[j].hi - x[u]) / d;
+        if (al < alpha) { alpha = al; blk = u; blk_up = true; }
+      }
+    }
+    if (blk >= 0) {  // blocked: step to the bound, fix the blocking variable
+#pragma unroll
+      for (int u = 0; u < V; ++u)
+        if (!((fix >> u) & 1u)) x[u] = pclamp(fma(alpha, xs[u] - x[u], x[u]), kc[u % N].lo, kc[u % N].hi);
+      x[blk] = blk_up ? kc[blk % N].hi : kc[blk % N].lo;
+      if (blk_up) up_m |= 1u << blk; else lo_m |= 1u << blk;
+      continue;
+    }
+#pragma unroll
+    for (int u = 0; u < V; ++u) x[u] = xs[u];
+    // stationary on the face: bound multipliers of the fixed variables
+    int worst = -1;
+    double most = -1e-12 * gscale;
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      if (!((fix >> u) & 1u)) continue;
+      double gr = g[u];
+#pragma unroll
+      for (int w = 0; w < V; ++w) gr = fma(move_h<N, M>(P, a, R, u, w), x[w], gr);
+      const double lam = ((lo_m >> u) & 1u) ? gr : -gr;
+      if (lam < most) { most = lam; worst = u; }
+    }
+    if (worst < 0) { status = 0u; break; }
+    lo_m &= ~(1u << worst);
+    up_m &= ~(1u << worst);
+  }
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+    uint32_t c = 0u;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const int v = t * N + j;
+      c |= ((((lo_m >> v) & 1u) ? 1u : 0u) | (((up_m >> v) & 1u) ? 2u : 0u)) << (2 * j);
+    }
+    act[t] = c;
+  }
+  return status;
 }
 
 // ------------------------------------------------------------------ S4 plant

@@ -58,6 +58,20 @@ struct RegArr {
   __device__ __forceinline__ void set(int t, double v) const { r[t] = v; }
 };
 
+// write-through accessor: reads the old value from `g`, writes the new one to
+// `g` and to a register copy (the per-period kernels' model push hands the
+// updated Sigma to the solve without re-reading it from memory)
+template <class A, int T>
+struct WriteThrough {
+  A g;
+  double (&c)[T];
+  __device__ __forceinline__ double get(int t) const { return g.get(t); }
+  __device__ __forceinline__ void set(int t, double v) const {
+    g.set(t, v);
+    c[t] = v;
+  }
+};
+
 // global-memory accessor for the per-period kernels (state in HBM)
 struct GlobAcc {
   double *p;
@@ -317,8 +331,8 @@ struct InstantOut {
 // roots s_t (warm starts for the next period), the per-block active codes and
 // the status; returns mean_j theta_j.  Only short-lived temporaries are kept
 // in registers (the caller's state lives in the slab / registers it owns).
-template <int N, int M, bool SCALED = false, bool SLO = false, class SAcc, class VAcc, class A0Acc, class TAcc,
-          class TmAcc>
+template <int N, int M, bool SCALED = false, bool SLO = false, bool MOVE = false, class SAcc, class VAcc,
+          class A0Acc, class TAcc, class TmAcc>
 __device__ __forceinline__ double control_instant(const DevParams &P, double inv_lam_k, double cap, double &w, VAcc mu_f,
                                                   double &mu_p, SAcc S, VAcc Sfp, A0Acc A0,
                                                   const double (&fbar)[N], double p, TAcc thr, TmAcc thr_max,
@@ -329,14 +343,21 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
   CAPGPU_PHASE_DECL
   // S1 (Eq. 5; Q1-Q4)
   double ahat[N];
-  model_push<N, SCALED>(P.lam, inv_lam_k, w, mu_f, mu_p, S, Sfp, fbar, p);
-  CAPGPU_MARK(P, 1, inst);
-  model_solve<N>(SCALED ? P.rho * inv_lam_k : P.rho, P.a_lo, P.a_hi, S, Sfp, A0, ahat);
+  if constexpr (SCALED) {
+    model_push<N, SCALED>(P.lam, inv_lam_k, w, mu_f, mu_p, S, Sfp, fbar, p);
+    CAPGPU_MARK(P, 1, inst);
+    model_solve<N>(P.rho * inv_lam_k, P.a_lo, P.a_hi, S, Sfp, A0, ahat);
+  } else {  // state in HBM: the solve takes the pushed Sigma from registers
+    double Sc[Tri<N>::size];
+    model_push<N, SCALED>(P.lam, inv_lam_k, w, mu_f, mu_p, WriteThrough<SAcc, Tri<N>::size>{S, Sc}, Sfp, fbar, p);
+    CAPGPU_MARK(P, 1, inst);
+    model_solve<N>(P.rho, P.a_lo, P.a_hi, RegArr<Tri<N>::size>{Sc}, Sfp, A0, ahat);
+  }
   CAPGPU_MARK(P, 2, inst);
   // S2: tau_j = ahat_j / R_j = ahat_j theta_j / r0_j.  theta only
   // feeds continuous quantities here, so it uses the fast reciprocal; the
   // reported theta and ranks (integers, bit-exact) use the IEEE division.
-  double tau[N], tsum0 = 0.0, tsum1 = 0.0;
+  double tau[N], thv[N], tsum0 = 0.0, tsum1 = 0.0;
   {
     double tr_[N], tm_[N];
 #pragma unroll
@@ -344,6 +365,7 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
       tr_[j] = thr.get(j);
       tm_[j] = thr_max.get(j);
       const double th = pclamp(tr_[j] * rcp_fast(tm_[j]), P.theta_min, 1.0);
+      thv[j] = th;
       if (j & 1) tsum1 += th; else tsum0 += th;
       tau[j] = ahat[j] * th * P.k[j].inv_r0;
     }
@@ -372,6 +394,26 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
   double beta = p - cap;
 #pragma unroll
   for (int j = 0; j < N; ++j) beta = fma(-ahat[j], fbar[j], beta);
+  if constexpr (MOVE) {  // NEXT-3: coupled blocks, generic active set (Q36)
+    double R[N], u[M * N], smin = 0.0, smax = 0.0;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      R[j] = P.k[j].r0 * rcp_fast(thv[j]);  // R_j = r0_j / theta_j (Q9)
+      smin = fma(ahat[j], P.k[j].lo, smin);
+      smax = fma(ahat[j], P.k[j].hi, smax);
+    }
+    status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
+    status |= move_qp<N, M>(P, P.k, ahat, R, beta, fbar, act, u);
+#pragma unroll
+    for (int j = 0; j < N; ++j) u0[j] = u[j];
+#pragma unroll
+    for (int t = 0; t < M; ++t) s_prev[t] = 0.0;
+    if (out.u) {
+#pragma unroll
+      for (int v = 0; v < M * N; ++v) out.u[(int64_t)v * out.ld] = u[v];
+    }
+    return tsum * P.inv_N;
+  }
   if (P.convex) {
     double smin = 0.0, smax = 0.0;
 #pragma unroll
@@ -562,8 +604,8 @@ struct SimOccupancy {
 
 // SLO: the NEXT-1 SLO-schedule instantiation (phase tracking, per-phase bounds,
 // miss counting); SLO-free runs use the SLO = false code, unchanged.
-template <int N, int M, int S, int BLOCK, bool SLO = false>
-__global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
+template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false>
+__global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 32 / BLOCK)
     k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
   using SL = SlabLayout<N>;
   extern __shared__ __align__(16) double smem[];
@@ -669,7 +711,7 @@ __global__ void __launch_bounds__(BLOCK, SimOccupancy<N>::warps * 32 / BLOCK)
       phase = slo_r >= P.slo_lo && slo_r < P.slo_hi ? 1 : 0;
       if (P.slo_period > 0 && ++slo_r == P.slo_period) slo_r = 0;
     }
-    const double tbar = control_instant<N, M, true, SLO>(P, inv_lam_k, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
+    const double tbar = control_instant<N, M, true, SLO, MOVE>(P, inv_lam_k, cap, w, MU, mu_p, Sm, SF, A0, fbar, p, RegArr<N>{thr}, TM, s_prev,
                                               act, u0, status, io, i, phase);
     CAPGPU_MARK(P, 0, i);
     if (slot >= 0) {
@@ -1023,10 +1065,63 @@ __device__ __forceinline__ void cta_sum2(double a, double b, double *out_a, doub
   }
 }
 
+// Servers per CTA of the per-period kernel (and of the S5 CTA partial sums:
+// 1024-server budget blocks are kBudgetBlock / kPeriodCta CTAs).  64: four
+// CTAs per SM (register and shared-memory limits at N = 9), so the stage-in,
+// compute and write-back phases of different CTAs overlap.
+#ifndef CAPGPU_PERIOD_CTA
+#define CAPGPU_PERIOD_CTA 64
+#endif
+constexpr int kPeriodCta = CAPGPU_PERIOD_CTA;
+
+// Per-warp SoA tile in shared memory (field-major, 32 lanes): k_period stages
+// the server's model state and read-only constants into it with cp.async at
+// the start of the period (one memory round trip per thread instead of one per
+// dependent use), then computes from it.  Lane accesses are consecutive 8-byte
+// words: conflict-free.
+struct TileAcc {
+  double *p;  // tile base + lane
+  __device__ __forceinline__ double get(int t) const { return p[t * 32]; }
+  __device__ __forceinline__ void set(int t, double v) const { p[t * 32] = v; }
+};
+
+template <int N>
+struct PeriodTile {
+  static constexpr int T = Tri<N>::size;
+  // Sigma | mu_f | Sfp | A0 | thr_max | base | amp; the read-only constants are
+  // staged only when the 128-thread tile fits the 227 KB of shared memory
+  // (N <= 15), else they are read from global memory where used.
+  static constexpr bool ro = (T + 6 * N) * kPeriodCta * 8 <= 227 * 1024;
+  static constexpr int oS = 0, oMU = T, oSFP = T + N, oA0 = T + 2 * N, oTM = T + 3 * N, oBA = T + 4 * N,
+                       oAM = T + 5 * N, F = ro ? T + 6 * N : T + 2 * N;
+  static constexpr int bytes_per_cta = F * kPeriodCta * 8;
+};
+
+template <bool RO>
+struct PeriodRo {
+  using type = TileAcc;
+  static __device__ __forceinline__ TileAcc make(double *tile, int o, const double *, int64_t, int64_t) {
+    return TileAcc{tile + o * 32};
+  }
+};
+template <>
+struct PeriodRo<false> {
+  using type = LdgAcc;
+  static __device__ __forceinline__ LdgAcc make(double *, int, const double *g, int64_t i, int64_t ld) {
+    return LdgAcc{g + i, ld};
+  }
+};
+
+__device__ __forceinline__ void cp_async8(double *smem_dst, const double *gsrc) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
 // One instant of the hierarchical configuration for every local server:
 // budget caps, S1-S3, the w_i / p partial sums, S4.  State in HBM.
-template <int N, int M>
-__global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
+template <int N, int M, int SS>
+__global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
                                                 int kk, int K) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = i < P.n_srv;
@@ -1042,20 +1137,38 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
   const double Br = fmin(Bmax, fma(bd.B_c - bd.pmin_tot, Wr / W, Pr));
   const double cap = fma(Br - Pr, w_prev / Wr, pmin_i);
   double tbar = 0.0, p = 0.0;
+  using PT = PeriodTile<N>;
+  extern __shared__ __align__(16) double ptile[];
+  double *tile = ptile + (threadIdx.x >> 5) * (PT::F * 32) + (threadIdx.x & 31);
   if (valid) {
-    double fbar[N], acc[N], thr[N], thr_max[N], mu_f[N], Sfp[N], A0r[N], base[N], amp[N];
+    // Stage Sigma, mu_f, Sfp and the read-only constants into this warp's tile
+    // (asynchronous, no registers held), load what crosses the period (fbar,
+    // acc, thr) into registers, then wait once.
+#pragma unroll
+    for (int t = 0; t < PT::T; ++t) cp_async8(tile + (PT::oS + t) * 32, st.S + t * ld + i);
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      cp_async8(tile + (PT::oMU + j) * 32, st.mu_f + j * ld + i);
+      cp_async8(tile + (PT::oSFP + j) * 32, st.Sfp + j * ld + i);
+      if constexpr (PT::ro) {
+        cp_async8(tile + (PT::oA0 + j) * 32, st.A0 + j * ld + i);
+        cp_async8(tile + (PT::oTM + j) * 32, st.thr_max + j * ld + i);
+        cp_async8(tile + (PT::oBA + j) * 32, st.base + j * ld + i);
+        cp_async8(tile + (PT::oAM + j) * 32, st.amp + j * ld + i);
+      }
+    }
+    double fbar[N], acc[N], thr[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       fbar[j] = st.fbar[j * ld + i];
       acc[j] = st.acc[j * ld + i];
       thr[j] = st.thr[j * ld + i];
-      thr_max[j] = st.thr_max[j * ld + i];
-      mu_f[j] = st.mu_f[j * ld + i];
-      Sfp[j] = st.Sfp[j * ld + i];
-      A0r[j] = st.A0[j * ld + i];
-      base[j] = st.base[j * ld + i];
-      amp[j] = st.amp[j * ld + i];
     }
+    cp_async_wait_all();
+    const TileAcc S{tile + PT::oS * 32}, MUF{tile + PT::oMU * 32}, SFP{tile + PT::oSFP * 32};
+    using RO = PeriodRo<PT::ro>;
+    const typename RO::type A0a = RO::make(tile, PT::oA0, st.A0, i, ld), TMa = RO::make(tile, PT::oTM, st.thr_max, i, ld),
+                            BAa = RO::make(tile, PT::oBA, st.base, i, ld), AMa = RO::make(tile, PT::oAM, st.amp, i, ld);
     double w = st.w[i], mu_p = st.mu_p[i];
     p = st.p[i];
     double s_prev[M];
@@ -1075,10 +1188,9 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
       io.theta = tr.theta ? tr.theta + (int64_t)kk * N * tr.n_trace + slot : nullptr;
       io.rank = tr.rank ? tr.rank + (int64_t)kk * N * tr.n_trace + slot : nullptr;
     }
-    const GlobAcc S{st.S + i, ld};
     double u0[N];
-    tbar = control_instant<N, M>(P, 0.0, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
-                                 RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
+    tbar = control_instant<N, M>(P, 0.0, cap, w, MUF, mu_p, S, SFP, A0a, fbar, p, RegArr<N>{thr}, TMa, s_prev, act,
+                                 u0, status, io);
     if (slot >= 0) {
       const int64_t b = (int64_t)kk * tr.n_trace + slot;
       if (tr.p) tr.p[b] = p;
@@ -1092,9 +1204,10 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
     // ---- S4: period k -> k+1
     const uint64_t srv = (uint64_t)(P.srv_begin + i);
     const uint32_t bm = burst_mask<N>(P, gen_stream_key(P.seed, GEN_TAG_BURST, srv), (k + 1) / GEN_BURST_HOLD);
-    double dem[N];
-    demand_all<N>(P, gen_stream_key(P.seed, GEN_TAG_JIT, srv), k + 1, bm, thr_max, RegArr<N>{base},
-                  RegArr<N>{amp}, dem);
+    double dem[N], thr_max[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) thr_max[j] = TMa.get(j);
+    demand_all<N>(P, gen_stream_key(P.seed, GEN_TAG_JIT, srv), k + 1, bm, thr_max, BAa, AMa, dem);
     if (slot >= 0 && tr.levels) {
       double u_l[N], a_l[N];
 #pragma unroll
@@ -1105,7 +1218,10 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
       plant_trace_levels<N>(P.k_dev, P.S, P.grid, u_l, a_l, tr.levels + (int64_t)kk * P.S * N * tr.n_trace + slot,
                             tr.n_trace);
     }
-    plant_delta_sigma<N>(P, P.grid, u0, acc, dem, thr_max, fbar, thr);
+    if constexpr (SS > 0)
+      plant_delta_sigma_c<N, SS>(P, P.grid, u0, acc, dem, thr_max, fbar, thr);
+    else
+      plant_delta_sigma<N>(P, P.grid, u0, acc, dem, thr_max, fbar, thr);
     const double noise = gen_noise(gen_stream_key(P.seed, GEN_TAG_NOISE, srv), k + 1, P.noise_scale);
     double pw = st.c_true[i];
 #pragma unroll
@@ -1134,9 +1250,11 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
       st.fbar[j * ld + i] = fbar[j];
       st.acc[j * ld + i] = acc[j];
       st.thr[j * ld + i] = thr[j];
-      st.mu_f[j * ld + i] = mu_f[j];
-      st.Sfp[j * ld + i] = Sfp[j];
+      st.mu_f[j * ld + i] = MUF.get(j);
+      st.Sfp[j * ld + i] = SFP.get(j);
     }
+#pragma unroll
+    for (int t = 0; t < PT::T; ++t) st.S[t * ld + i] = S.get(t);
     st.w[i] = w;
     st.mu_p[i] = mu_p;
     st.p[i] = p_next;
@@ -1148,7 +1266,7 @@ __global__ void __launch_bounds__(128) k_period(DevParams P, StatePtrs st, Budge
     bd.srv_w[i] = tbar;
   }
   const int n_cta = gridDim.x;
-  cta_sum2<128>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
+  cta_sum2<kPeriodCta>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
 }
 
 // w_i(0) = mean_j theta_ij(0) of the initial state, its CTA partials, and the
@@ -1176,9 +1294,9 @@ __global__ void __launch_bounds__(128) k_budget_init(DevParams P, StatePtrs st, 
     p = st.p[i];
   }
   const int n_cta = gridDim.x;
-  cta_sum2<128>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
+  cta_sum2<kPeriodCta>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
   __syncthreads();
-  cta_sum2<128>(pmn, pmx, &cta_part_c[blockIdx.x], &cta_part_c[n_cta + blockIdx.x]);
+  cta_sum2<kPeriodCta>(pmn, pmx, &cta_part_c[blockIdx.x], &cta_part_c[n_cta + blockIdx.x]);
 }
 
 // ------------------------------------------------------------------ control step (per-period mode)
@@ -1369,7 +1487,7 @@ struct LaunchN {
   }
   static int budget_init(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, double *part_c,
                          cudaStream_t s) {
-    k_budget_init<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, bd, part_c);
+    k_budget_init<N><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, 0, s>>>(P, st, bd, part_c);
     return (int)cudaGetLastError();
   }
 };
@@ -1377,13 +1495,17 @@ struct LaunchN {
 // Fused-kernel launch: block size chosen so that the last wave is nearly full
 // (the per-instance period chain is serial, so a ragged last wave costs a
 // whole per-instance run time).
-template <int N, int M, int S, int BLOCK, bool SLO = false>
+template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false>
 int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
   const int smem = (int)(sizeof(double) * SlabLayout<N>::F * BLOCK);
-  cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK, SLO>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  k_simulate<N, M, S, BLOCK, SLO><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
+  cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK, SLO, MOVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  k_simulate<N, M, S, BLOCK, SLO, MOVE><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
   return (int)cudaGetLastError();
 }
+
+// NEXT-3 move-suppressed QP: instantiated for the stacked sizes the per-thread
+// dense active set holds in registers (M N <= kMoveMaxVars)
+constexpr int kMoveMaxVars = 10;
 
 template <int N, int M, int S>
 int sim_occupancy(int block, int n_class) {
@@ -1435,6 +1557,10 @@ struct LaunchNM {
       const double nb = std::ceil((double)P.n_inst / block);
       return std::ceil(nb / sms) * block * (1.0 + 0.02 * (8.0 / (occ * block / 32.0)));
     };
+    if (P.wmove > 0.0) {  // NEXT-3 (one block size; validated: no SLO schedule, M N <= kMoveMaxVars)
+      if constexpr (N * M <= kMoveMaxVars) return launch_sim<N, M, S, 32, false, true>(P, st, tr, k0, K, s);
+      return (int)cudaErrorInvalidConfiguration;
+    }
     if (P.slo) return launch_sim<N, M, S, 32, true>(P, st, tr, k0, K, s);  // NEXT-1 (one block size)
     if (occ128[nc] <= 0 || busiest(occ32[nc], 32) < busiest(occ128[nc], 128))
       return launch_sim<N, M, S, 32>(P, st, tr, k0, K, s);
@@ -1454,7 +1580,14 @@ struct LaunchNM {
   }
   static int period(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, const TracePtrs &tr, int64_t k,
                     int kk, int K, cudaStream_t s) {
-    k_period<N, M><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, bd, tr, k, kk, K);
+    const int smem = PeriodTile<N>::bytes_per_cta;
+    if (P.S == 4) {
+      cudaFuncSetAttribute(k_period<N, M, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      k_period<N, M, 4><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, smem, s>>>(P, st, bd, tr, k, kk, K);
+    } else {
+      cudaFuncSetAttribute(k_period<N, M, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      k_period<N, M, 0><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, smem, s>>>(P, st, bd, tr, k, kk, K);
+    }
     return (int)cudaGetLastError();
   }
 };
