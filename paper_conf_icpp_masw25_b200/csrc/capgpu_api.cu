@@ -7,6 +7,7 @@
 // and launches.
 #include <cmath>
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -291,8 +292,9 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   const int64_t nd_inst = (int64_t)(5 * N + c->T + 4);
   const int64_t nd_srv = (int64_t)(5 * N + 3);
   const int64_t grid_bytes = (int64_t)sizeof(GridEntry) * n_class * CAPGPU_MAX_LEVELS;
-  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 12 * (int64_t)h.M * ni + 4 * ni + grid_bytes +
-                        (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS * 3 + 256;
+  const int64_t sched_words = ni + 2;  // chunked schedule of the fused kernel: counter + done[instance]
+  const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 12 * (int64_t)h.M * ni + 4 * ni + 4 * sched_words +
+                        grid_bytes + (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS * 3 + 256;
   cudaError_t e = cudaMalloc(&c->ws, (size_t)bytes);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -333,6 +335,11 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   d.k_dev_slo[1] = c->kdev_slo + CAPGPU_MAX_KNOBS;
   s.trace_slot = (int32_t *)q;
   s.act = (uint32_t *)(s.trace_slot + ni);
+  s.sched = (int32_t *)(s.act + (int64_t)h.M * ni);
+  {
+    const char *nc = getenv("CAPGPU_NO_CHUNKING");
+    d.no_chunking = (nc && nc[0] && nc[0] != '0') ? 1 : 0;
+  }
   for (int c2 = 0; c2 < n_class; ++c2)
     cudaMemcpy(gdev + c2 * CAPGPU_MAX_LEVELS, grid[c2], sizeof(GridEntry) * CAPGPU_MAX_LEVELS,
                cudaMemcpyHostToDevice);

@@ -92,6 +92,7 @@ struct DevParams {
   int32_t bl_kind, bl_steps;
   double bl_margin, bl_pole;
   double wmove;              // NEXT-3 move-suppression weight W (Q36); 0 = the literal Eq. 9
+  int32_t no_chunking;       // 1: fused kernel without the chunked persistent schedule (env CAPGPU_NO_CHUNKING)
   long long *phase;          // [8][n_inst] cycle counters (builds with -DCAPGPU_PHASE_TIMING only)
   KnobConst k[kMaxN];
 };

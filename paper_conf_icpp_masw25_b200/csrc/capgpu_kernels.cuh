@@ -12,6 +12,7 @@
 //   k_assign_weights S2 alone
 #pragma once
 
+#include <algorithm>
 #include <cmath>
 
 #include "capgpu_device.cuh"
@@ -29,6 +30,7 @@ struct StatePtrs {
   uint32_t *act;                           // [M] warm-start active codes of the block QPs
   double *cap_base;                        // [1]
   int32_t *trace_slot;                     // [1] -1 = not traced
+  int32_t *sched;                          // chunked schedule: counter + per-instance done flags (n_inst + 2)
   // per server (ld = n_srv)
   double *a_true, *c_true, *thr_max, *base, *amp, *A0, *pmin, *pmax;
 };
@@ -604,17 +606,76 @@ struct SimOccupancy {
 
 // SLO: the NEXT-1 SLO-schedule instantiation (phase tracking, per-phase bounds,
 // miss counting); SLO-free runs use the SLO = false code, unchanged.
-template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false>
-__global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 32 / BLOCK)
-    k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
+//
+// sim_run: instance i advanced over periods k0 .. k0 + K - 1, which are the
+// call's periods kk0 .. kk0 + K - 1 of Ktot (trace rows and the summary window
+// are indexed by the call's period).  carry: a later chunk of the same call
+// (the running summaries are read back from the trace arrays).  Mutable state
+// and summaries move with L1-bypassing loads/stores (ld/st.cg): another SM may
+// run the instance's next chunk.
+// Chunked schedule (SimSched.ctr != nullptr): the call's periods are cut into
+// C chunks and the work items (CTA group g, chunk c) are handed out c-major
+// from a global counter as CTAs start, so every resident slot stays busy until
+// the last round.  Without it, n_inst instances on R resident slots take
+// ceil(n_inst / R) full runs of K periods (cfg 3: 65 536 instances on 37 888
+// slots = 1.73 runs of work in 2 run times).  Instance i of item (g, c) waits
+// for done[i] >= the chunk's first period (release/acquire at gpu scope, one
+// flag per instance: no CTA barrier or fence after the period loop).
+struct SimSched {
+  int32_t *ctr;   // [1] next item (zeroed before the launch)
+  int32_t *done;  // [n_inst] call periods completed per instance (zeroed before the launch)
+  int32_t n_groups, Kc, n_items;
+};
+
+__device__ __forceinline__ int ld_acquire_gpu(const int32_t *p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(int32_t *p, int v) {
+  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// The work item (instance, chunk) is re-derived from the item in shared memory
+// and the kernel parameters (constant bank) at stage-in and again at
+// stage-out: nothing of the schedule stays live in registers across the loop.
+struct SimChunk {
+  int64_t i;   // instance
+  int kk0, K;  // the chunk's first call period and its period count
+};
+// CH = false: one item per CTA (blockIdx), all Ktot periods -- the plain
+// launch, compiled without any of the schedule's state.
+template <int BLOCK, bool CH>
+__device__ __forceinline__ SimChunk sim_chunk(const SimSched &sc, const int *item_sh, int Ktot) {
+  if constexpr (!CH) {
+    (void)sc;
+    (void)item_sh;
+    return SimChunk{(int64_t)blockIdx.x * BLOCK + threadIdx.x, 0, Ktot};
+  } else {
+    const int it = *(const volatile int *)item_sh;
+    const int c = it / sc.n_groups;
+    const int kk0 = c * sc.Kc;
+    return SimChunk{(int64_t)(it - c * sc.n_groups) * BLOCK + threadIdx.x, kk0, min(sc.Kc, Ktot - kk0)};
+  }
+}
+
+template <int N, int M, int S, int BLOCK, bool SLO, bool MOVE, bool CH>
+__device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st, const TracePtrs &tr,
+                                        const SimSched &sc, const int *item_sh, const int64_t &k0call,
+                                        const int &Ktot, double *my) {
   using SL = SlabLayout<N>;
-  extern __shared__ __align__(16) double smem[];
+  const SimChunk ck = sim_chunk<BLOCK, CH>(sc, item_sh, Ktot);
+  int64_t i = ck.i;
+  const int kk0 = ck.kk0, K = ck.K;
+  const int64_t k0 = k0call + kk0;
+  const bool carry = CH && kk0 > 0;
+  // chunked schedule: wait until the previous chunk of this instance has
+  // written its state back (done[i] = call periods done, release/acquire)
+  if (carry)
+    while (ld_acquire_gpu(sc.done + i) < kk0) __nanosleep(128);
   // grid tables: read-only global (L1-resident, 1 KB per class) so the whole
   // shared memory goes to the per-thread slabs
   const GridEntry *sgrid = P.grid;
-  int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x;
-  if (i >= P.n_inst) return;
-  double *my = smem + threadIdx.x * SL::F;
   const Slab Sm{my};
   const Slab MU{my + SL::oMU};
   const Slab SF{my + SL::oSFP};
@@ -637,11 +698,11 @@ __global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 3
   double fbar[N], acc[N], thr[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    fbar[j] = st.fbar[j * li + i];
-    acc[j] = st.acc[j * li + i];
-    thr[j] = st.thr[j * li + i];
-    MU.set(j, st.mu_f[j * li + i]);
-    SF.set(j, st.Sfp[j * li + i]);
+    fbar[j] = __ldcg(st.fbar + j * li + i);
+    acc[j] = __ldcg(st.acc + j * li + i);
+    thr[j] = __ldcg(st.thr + j * li + i);
+    MU.set(j, __ldcg(st.mu_f + j * li + i));
+    SF.set(j, __ldcg(st.Sfp + j * li + i));
     if constexpr (!SL::ro_global) {
       my[SL::oA0 + j] = st.A0[j * ls + si];
       my[SL::oAT + j] = __dmul_rn(gain, st.a_true[j * ls + si]);
@@ -651,16 +712,16 @@ __global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 3
     }
   }
 #pragma unroll
-  for (int t = 0; t < SL::T; ++t) Sm.set(t, st.S[t * li + i]);
-  double p = st.p[i], w = st.w[i], mu_p = st.mu_p[i];
+  for (int t = 0; t < SL::T; ++t) Sm.set(t, __ldcg(st.S + t * li + i));
+  double p = __ldcg(st.p + i), w = __ldcg(st.w + i), mu_p = __ldcg(st.mu_p + i);
   const double c_true = st.c_true[si], cap_base = st.cap_base[i];
   double s_prev[M];
 #pragma unroll
   uint32_t act[M];
 #pragma unroll
   for (int t = 0; t < M; ++t) {
-    s_prev[t] = st.s_prev[t * li + i];
-    act[t] = st.act[t * li + i];
+    s_prev[t] = __ldcg(st.s_prev + t * li + i);
+    act[t] = __ldcg(st.act + t * li + i);
   }
   const int slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
   const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
@@ -672,22 +733,33 @@ __global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 3
   uint32_t bmask = burst_mask<N>(P, kburst, epoch);
 
   // ---- summaries (Q25)
-  const int kw = K - (4 * K) / 5;
+  const int kw = Ktot - (4 * Ktot) / 5;
   double sum_p = 0.0, sumsq_p = 0.0, max_p = 0.0, sum_theta = 0.0;
   int n_viol = 0, n_miss = 0;
+  if (carry) {
+    if (tr.sum_p) sum_p = __ldcg(tr.sum_p + i);
+    if (tr.sumsq_p) sumsq_p = __ldcg(tr.sumsq_p + i);
+    if (tr.max_p) max_p = __ldcg(tr.max_p + i);
+    if (tr.sum_theta) sum_theta = __ldcg(tr.sum_theta + i);
+    if (tr.n_viol) n_viol = __ldcg(tr.n_viol + i);
+    if (tr.n_miss) n_miss = __ldcg(tr.n_miss + i);
+  }
   // SLO schedule position r = k mod slo_period (NEXT-1), advanced per period
   int64_t slo_r = SLO && P.slo_period > 0 ? k0 % P.slo_period : 0;
   int act_cnt[M];
 #pragma unroll
-  for (int t = 0; t < M; ++t) act_cnt[t] = 0;
+  for (int t = 0; t < M; ++t) act_cnt[t] = carry && tr.act_count ? __ldcg(tr.act_count + t * li + i) : 0;
 
   // the slab holds Sigma' = Sigma / lam^kk (model_push SCALED); inv_lam_k = lam^-kk
   double inv_lam_k = 1.0;
 
   CAPGPU_PHASE_DECL
+  // the loop bound is read from shared memory (item_sh[1], the same for the
+  // whole CTA) each period instead of occupying a register across the loop
+  (void)K;
 #pragma unroll 1
-  for (int kk = 0; kk < K; ++kk) {
-    const int64_t k = k0 + kk;
+  for (int kk = kk0; kk < (CH ? *(const volatile int *)(item_sh + 1) : Ktot); ++kk) {  // the call's period
+    const int64_t k = k0call + kk;
     const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
     if ((kk & 1023) == 1023) {  // keep lam^-kk far from overflow: fold it back into Sigma'
       slab_rescale<N>(my, SL::oSFP, rcp_fast(inv_lam_k));
@@ -780,37 +852,70 @@ __global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 3
   // ---- write back.  Launder the indices so the compiler recomputes the ~100
   // state addresses here instead of keeping the stage-in ones alive (spilled)
   // across the whole period loop.
+  const SimChunk ck2 = sim_chunk<BLOCK, CH>(sc, item_sh, Ktot);
+  i = ck2.i;
+  si = i / P.n_caps;
+  li = P.n_inst;
+  ls = P.n_srv;
   asm volatile("" : "+l"(i), "+l"(li), "+l"(ls), "+l"(si));
   const double lam_k = rcp_fast(inv_lam_k);  // Sigma = lam^kk Sigma'
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    st.fbar[j * li + i] = fbar[j];
-    st.acc[j * li + i] = acc[j];
-    st.thr[j * li + i] = thr[j];
-    st.mu_f[j * li + i] = MU.get(j);
-    st.Sfp[j * li + i] = SF.get(j) * lam_k;
+    __stcg(st.fbar + j * li + i, fbar[j]);
+    __stcg(st.acc + j * li + i, acc[j]);
+    __stcg(st.thr + j * li + i, thr[j]);
+    __stcg(st.mu_f + j * li + i, MU.get(j));
+    __stcg(st.Sfp + j * li + i, SF.get(j) * lam_k);
   }
 #pragma unroll
-  for (int t = 0; t < SL::T; ++t) st.S[t * li + i] = Sm.get(t) * lam_k;
-  st.p[i] = p;
-  st.w[i] = w;
-  st.mu_p[i] = mu_p;
+  for (int t = 0; t < SL::T; ++t) __stcg(st.S + t * li + i, Sm.get(t) * lam_k);
+  __stcg(st.p + i, p);
+  __stcg(st.w + i, w);
+  __stcg(st.mu_p + i, mu_p);
 #pragma unroll
   for (int t = 0; t < M; ++t) {
-    st.s_prev[t * li + i] = s_prev[t];
-    st.act[t * li + i] = act[t];
+    __stcg(st.s_prev + t * li + i, s_prev[t]);
+    __stcg(st.act + t * li + i, act[t]);
   }
-  if (tr.sum_p) tr.sum_p[i] = sum_p;
-  if (tr.sumsq_p) tr.sumsq_p[i] = sumsq_p;
-  if (tr.max_p) tr.max_p[i] = max_p;
-  if (tr.sum_theta) tr.sum_theta[i] = sum_theta;
-  if (tr.n_viol) tr.n_viol[i] = n_viol;
-  if (tr.n_miss) tr.n_miss[i] = n_miss;
-  if (tr.n_window) tr.n_window[i] = K - kw;
+  if (tr.sum_p) __stcg(tr.sum_p + i, sum_p);
+  if (tr.sumsq_p) __stcg(tr.sumsq_p + i, sumsq_p);
+  if (tr.max_p) __stcg(tr.max_p + i, max_p);
+  if (tr.sum_theta) __stcg(tr.sum_theta + i, sum_theta);
+  if (tr.n_viol) __stcg(tr.n_viol + i, n_viol);
+  if (tr.n_miss) __stcg(tr.n_miss + i, n_miss);
+  if (tr.n_window) tr.n_window[i] = Ktot - (Ktot - (4 * Ktot) / 5);
   if (tr.final_p) tr.final_p[i] = p;
   if (tr.act_count) {
 #pragma unroll
-    for (int t = 0; t < M; ++t) tr.act_count[t * li + i] = act_cnt[t];
+    for (int t = 0; t < M; ++t) __stcg(tr.act_count + t * li + i, act_cnt[t]);
+  }
+  if constexpr (CH) st_release_gpu(sc.done + i, ck2.kk0 + ck2.K);  // orders this thread's state stores before it
+}
+
+template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false, bool CH = false>
+__global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 32 / BLOCK)
+    k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K, SimSched sc) {
+  extern __shared__ __align__(16) double smem[];
+  double *my = smem + threadIdx.x * SlabLayout<N>::F;
+  if constexpr (!CH) {
+    if ((int64_t)blockIdx.x * BLOCK + threadIdx.x < P.n_inst)
+      sim_run<N, M, S, BLOCK, SLO, MOVE, false>(P, st, tr, sc, nullptr, k0, K, my);
+  } else {
+    // one CTA per work item, the item taken from the counter when the CTA
+    // starts (the dynamic-tile-id order), so item (g, c - 1) belongs to a CTA
+    // that started earlier and is resident or done: the per-instance waits in
+    // sim_run always end.
+    __shared__ int item_s[2];  // work item, end of its period range (call periods)
+    if (threadIdx.x == 0) {
+      const int it = atomicAdd(sc.ctr, 1);
+      item_s[0] = it;
+      item_s[1] = min((it / sc.n_groups + 1) * sc.Kc, K);
+    }
+    __syncthreads();
+    const int item = item_s[0];
+    const int c = item / sc.n_groups, g = item - c * sc.n_groups;
+    if ((int64_t)g * BLOCK + threadIdx.x < P.n_inst)
+      sim_run<N, M, S, BLOCK, SLO, MOVE, true>(P, st, tr, sc, item_s, k0, K, my);
   }
 }
 
@@ -1495,11 +1600,65 @@ struct LaunchN {
 // Fused-kernel launch: block size chosen so that the last wave is nearly full
 // (the per-instance period chain is serial, so a ragged last wave costs a
 // whole per-instance run time).
+//
+// With more instance groups than resident slots the call runs the chunked
+// persistent schedule (SimSched): C chunks of the K periods, C chosen so the
+// item count n_groups * C fills whole rounds of the resident slots (the last
+// round's idle fraction is what the schedule cannot recover) while the
+// per-chunk state round trip (~2 KB per instance) stays small against a chunk.
+inline int sim_chunks(int64_t n_groups, int64_t slots, int K) {
+  if (n_groups <= slots || K < 64) return 1;
+  int best = 1;
+  const double r1 = (double)n_groups / slots;
+  double best_cost = (std::ceil(r1) - r1) / std::ceil(r1);  // C = 1: the plain launch
+  for (int C = 2; C <= 64 && K / C >= 16; ++C) {
+    const double rounds = (double)n_groups * C / slots;
+    const double idle = (std::ceil(rounds) - rounds) / std::ceil(rounds);  // last-round idle share
+    const double cost = idle + 0.002 * C;                                    // + state round trips
+    if (cost < best_cost) {
+      best_cost = cost;
+      best = C;
+    }
+  }
+  return best;
+}
+
 template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false>
 int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
   const int smem = (int)(sizeof(double) * SlabLayout<N>::F * BLOCK);
-  cudaFuncSetAttribute(k_simulate<N, M, S, BLOCK, SLO, MOVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  k_simulate<N, M, S, BLOCK, SLO, MOVE><<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K);
+  // the chunked schedule is instantiated for the plain CapGPU kernel (no SLO
+  // schedule, no move suppression, compile-time S) with 32-wide CTAs
+  constexpr bool can_chunk = !SLO && !MOVE && S > 0 && BLOCK == 32;
+  int C = 1;
+  const int64_t n_groups = (P.n_inst + BLOCK - 1) / BLOCK;
+  if constexpr (can_chunk) {
+    auto kc = k_simulate<N, M, S, BLOCK, false, false, true>;
+    int occ = 0, dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kc, BLOCK, smem) != cudaSuccess) {
+      cudaGetLastError();
+      occ = 0;
+    }
+    const int64_t slots = (int64_t)occ * sms;
+    C = (st.sched && slots > 0 && !P.no_chunking) ? sim_chunks(n_groups, slots, K) : 1;
+    if (C > 1) {
+      SimSched sc{};
+      sc.ctr = st.sched;
+      sc.done = st.sched + 1;
+      sc.n_groups = (int32_t)n_groups;
+      sc.Kc = (K + C - 1) / C;
+      sc.n_items = (int32_t)(n_groups * ((K + sc.Kc - 1) / sc.Kc));
+      cudaError_t e = cudaMemsetAsync(st.sched, 0, sizeof(int32_t) * (size_t)(P.n_inst + 1), s);
+      if (e != cudaSuccess) return (int)e;
+      kc<<<(unsigned)sc.n_items, BLOCK, smem, s>>>(P, st, tr, k0, K, sc);
+      return (int)cudaGetLastError();
+    }
+  }
+  auto kern = k_simulate<N, M, S, BLOCK, SLO, MOVE>;
+  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  kern<<<grid_for(P.n_inst, BLOCK), BLOCK, smem, s>>>(P, st, tr, k0, K, SimSched{});
   return (int)cudaGetLastError();
 }
 

@@ -279,7 +279,45 @@ def test_closed_loop_cfg3_full_size(G, oracle_mod):
     bench's launch configuration; 24 sampled servers compared element by element."""
     d = configs.get(3)
     tr = np.linspace(0, 65535, 24).astype(np.int64)
-    _sim_compare(G, oracle_mod, d, 65536, tr)
+    _, gp, ref = _sim_compare(G, oracle_mod, d, 65536, tr)
+    _summary_compare(gp, ref["summary"], tr)
+
+
+def _summary_compare(gp, s, idx):
+    """Per-instance summaries (window sums, max, violations, active-set counts):
+    carried across the chunks of the persistent schedule."""
+    n_win = s["n_window"]
+    np.testing.assert_allclose(gp["sum_p"][idx], s["sum_p"], rtol=0, atol=1e-6 * n_win.max())
+    np.testing.assert_allclose(gp["max_p"][idx], s["max_p"], rtol=0, atol=1e-6)
+    np.testing.assert_allclose(gp["sum_theta"][idx], s["sum_theta"], rtol=1e-9)
+    assert np.array_equal(gp["n_viol"][idx], s["n_viol"])
+    assert np.array_equal(gp["n_window"][idx], n_win)
+    assert np.array_equal(gp["act_count"][:, idx].T, s["act_count"])
+
+
+def test_chunked_schedule_matches_single_pass(G, oracle_mod, monkeypatch):
+    """The chunked persistent schedule (more instance groups than resident slots,
+    DESIGN.md §5) against the one-item-per-CTA launch of the same call: every
+    instance's summaries and final power agree to rounding (the chunk boundary
+    re-scales the model state, 1e-16 relative), sampled instances match the
+    oracle including the summaries carried across chunks."""
+    d = configs.get(3)
+    n, K = 65536, 200
+    wl = G.workload_from(d)
+    monkeypatch.setenv("CAPGPU_NO_CHUNKING", "1")
+    g1 = G.CapGPU.from_config(d, n_servers=n)
+    monkeypatch.delenv("CAPGPU_NO_CHUNKING")
+    one = {k: H(v) for k, v in g1.simulate(K, wl).items()}
+    del g1
+    tr = np.array([0, 777, 40000, 65535])
+    g2 = G.CapGPU.from_config(d, n_servers=n)
+    ch = {k: H(v) for k, v in g2.simulate(K, wl, trace_inst=tr).items()}
+    np.testing.assert_allclose(ch["final_p"], one["final_p"], rtol=0, atol=1e-6)
+    np.testing.assert_allclose(ch["sum_p"], one["sum_p"], rtol=0, atol=1e-6 * K)
+    assert np.mean(ch["n_viol"] == one["n_viol"]) >= 0.9999
+    ref = oracle_mod.Oracle(d).simulate(tr, periods=K)
+    np.testing.assert_allclose(ch["tr_p"], ref["p"], rtol=0, atol=1e-6)
+    _summary_compare(ch, ref["summary"], tr)
 
 
 @pytest.mark.slow
