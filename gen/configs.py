@@ -17,7 +17,8 @@ GPU_KNOB = dict(f_min=435.0, f_max=1350.0, n_levels=11, sweep_base=0)   # base =
 
 # Controller constants (Q1, Q4, Q6, Q8, Q21; P = 8 / M = 2 from P:264; gamma P:190)
 CONTROLLER = dict(q=1.0, r0=1e-4, theta_min=0.05, lam=0.95, rho=100.0, a_lo=0.25, a_hi=4.0,
-                  a_floor=1e-3, gamma=0.91, noise_std=11.0, substeps=4, wmove=0.0)
+                  a_floor=1e-3, gamma=0.91, noise_std=11.0, substeps=4, wmove=0.0,
+                  ref_alpha=0.0)
 
 _BASE_WORKLOAD = dict(n_caps=1, demand_kind=1, demand_frac=0.7, cap_frac0=0.5, cap_frac_rand=0.0,
                       cap_frac_step=0.0, cap_period=0, cap_lo=0, cap_hi=0, cap_mult=1.0,

@@ -47,6 +47,7 @@ typedef struct {
   double noise_std;  /* meter noise sigma (W) */
   uint64_t seed;
   double wmove;      /* NEXT-3 move suppression weight W (W^2/MHz^2, Q36); 0 = the literal Eq. 9 */
+  double ref_alpha;  /* NEXT-3 reference trajectory alpha = exp(-T/T_ref) in [0, 1) (Q37); 0 = off */
 } ora_cfg;
 
 typedef struct {
@@ -139,6 +140,24 @@ double ora_mpc_cost(const ora_cfg *c, const double *Ahat, const double *R, doubl
 void ora_mpc_classify(const ora_cfg *c, const double *Ahat, const double *R, double beta,
                       const double *lo, const double *hi, const double *m, const double *u,
                       uint32_t *active, uint32_t *tie);
+/* NEXT-3 reference trajectory (Q37): row i of the tracking term has the
+ * offset beta + alpha^i dref, dref = P_s - p(k), alpha = cfg ref_alpha. */
+double ora_ref_pow(const ora_cfg *c, int i);
+double ora_mpc_cost_ref(const ora_cfg *c, const double *Ahat, const double *R, double beta, double dref,
+                        const double *m, const double *u);
+double ora_mpc_move_cost_ref(const ora_cfg *c, const double *Ahat, const double *R, double beta, double dref,
+                             const double *fbar, const double *m, const double *u);
+void ora_mpc_classify_ref(const ora_cfg *c, const double *Ahat, const double *R, double beta, double dref,
+                          const double *lo, const double *hi, const double *m, const double *u,
+                          uint32_t *active, uint32_t *tie);
+int ora_mpc_stacked_ref(const ora_cfg *c, const double *Ahat, const double *R, double beta, double dref,
+                        const double *lo, const double *hi, const double *m, double *u,
+                        uint32_t *active, uint32_t *tie, int *iters);
+int ora_mpc_move_ref(const ora_cfg *c, const double *Ahat, const double *R, double beta, double dref,
+                     const double *fbar, const double *lo, const double *hi, const double *m, double *u,
+                     uint32_t *active, uint32_t *tie, int *iters);
+int ora_mpc_bruteforce_ref(const ora_cfg *c, const double *Ahat, const double *R, double beta, double dref,
+                           const double *fbar, const double *lo, const double *hi, const double *m, double *u);
 
 /* ---- S4 plant (P:242 delta-sigma, P:238/P:264 meter, Eq. 5, Eq. 8/10b) */
 void ora_plant_step(const ora_cfg *c, const double *a_true, double c_true, const double *thr_max,

@@ -47,7 +47,7 @@ class OraCfg(C.Structure):
                 ("q", C.c_double), ("theta_min", C.c_double), ("lam", C.c_double),
                 ("rho", C.c_double), ("a_lo", C.c_double), ("a_hi", C.c_double),
                 ("a_floor", C.c_double), ("gamma", C.c_double), ("noise_std", C.c_double),
-                ("seed", C.c_uint64), ("wmove", C.c_double)]
+                ("seed", C.c_uint64), ("wmove", C.c_double), ("ref_alpha", C.c_double)]
 
 
 class OraWorkload(C.Structure):
@@ -107,6 +107,17 @@ def lib():
         L.ora_mpc_cost.argtypes = [cp, dp, dp, C.c_double, dp, dp]
         L.ora_mpc_cost.restype = C.c_double
         L.ora_mpc_classify.argtypes = [cp, dp, dp, C.c_double, dp, dp, dp, dp, u32p, u32p]
+        # NEXT-3 reference trajectory (Q37): the same with the offset dref = P_s - p(k)
+        L.ora_ref_pow.argtypes = [cp, C.c_int]
+        L.ora_ref_pow.restype = C.c_double
+        L.ora_mpc_stacked_ref.argtypes = [cp, dp, dp, C.c_double, C.c_double, dp, dp, dp, dp, u32p, u32p, ip]
+        L.ora_mpc_move_ref.argtypes = [cp, dp, dp, C.c_double, C.c_double, dp, dp, dp, dp, dp, u32p, u32p, ip]
+        L.ora_mpc_bruteforce_ref.argtypes = [cp, dp, dp, C.c_double, C.c_double, dp, dp, dp, dp, dp]
+        L.ora_mpc_cost_ref.argtypes = [cp, dp, dp, C.c_double, C.c_double, dp, dp]
+        L.ora_mpc_cost_ref.restype = C.c_double
+        L.ora_mpc_move_cost_ref.argtypes = [cp, dp, dp, C.c_double, C.c_double, dp, dp, dp]
+        L.ora_mpc_move_cost_ref.restype = C.c_double
+        L.ora_mpc_classify_ref.argtypes = [cp, dp, dp, C.c_double, C.c_double, dp, dp, dp, dp, u32p, u32p]
         L.ora_plant_step.argtypes = [cp, dp, C.c_double, dp, dp, C.c_double, dp, dp, dp, dp, dp,
                                      C.POINTER(C.c_uint8)]
         L.ora_gen_server.argtypes = [cp, C.c_uint64, dp, dp, dp, dp, dp]
@@ -159,6 +170,7 @@ def make_cfg(desc: dict) -> OraCfg:
     c.gamma, c.noise_std = ctl["gamma"], ctl["noise_std"]
     c.seed = desc["seed"]
     c.wmove = ctl.get("wmove", 0.0)
+    c.ref_alpha = ctl.get("ref_alpha", 0.0)
     return c
 
 
@@ -269,25 +281,28 @@ class Oracle:
         self.L.ora_block_weights(C.byref(self.cfg), _dp(ct))
         return ct
 
-    def mpc(self, Ahat, R, beta, lo, hi, m):
+    def mpc(self, Ahat, R, beta, lo, hi, m, dref=0.0):
+        """Eq. 9-10a as one dense stacked QP; dref = P_s - p(k) feeds the
+        reference trajectory when cfg ref_alpha > 0 (NEXT-3, Q37)."""
         Ahat, R, lo, hi, m = map(_arr, (Ahat, R, lo, hi, m))
         u = np.zeros((self.M, self.n))
         act = np.zeros(self.M, dtype=np.uint32); tie = np.zeros(self.M, dtype=np.uint32)
         it = np.zeros(1, dtype=np.int32)
-        st = self.L.ora_mpc_stacked(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(lo),
-                                    _dp(hi), _dp(m), _dp(u),
+        st = self.L.ora_mpc_stacked_ref(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), float(dref), _dp(lo),
+                                        _dp(hi), _dp(m), _dp(u),
                                     act.ctypes.data_as(C.POINTER(C.c_uint32)),
                                     tie.ctypes.data_as(C.POINTER(C.c_uint32)),
                                     it.ctypes.data_as(C.POINTER(C.c_int32)))
         return u, act, tie, int(st), int(it[0])
 
-    def mpc_move(self, Ahat, R, beta, fbar, lo, hi, m):
+    def mpc_move(self, Ahat, R, beta, fbar, lo, hi, m, dref=0.0):
         """NEXT-3: Eq. 9 + move suppression (cfg wmove), dense generic active set."""
         Ahat, R, fbar, lo, hi, m = map(_arr, (Ahat, R, fbar, lo, hi, m))
         u = np.zeros((self.M, self.n))
         act = np.zeros(self.M, dtype=np.uint32); tie = np.zeros(self.M, dtype=np.uint32)
         it = np.zeros(1, dtype=np.int32)
-        st = self.L.ora_mpc_move(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(fbar), _dp(lo), _dp(hi),
+        st = self.L.ora_mpc_move_ref(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), float(dref), _dp(fbar),
+                                     _dp(lo), _dp(hi),
                                  _dp(m), _dp(u), act.ctypes.data_as(C.POINTER(C.c_uint32)),
                                  tie.ctypes.data_as(C.POINTER(C.c_uint32)), it.ctypes.data_as(C.POINTER(C.c_int32)))
         return u, act, tie, int(st), int(it[0])
@@ -305,23 +320,28 @@ class Oracle:
         Ahat, R, fbar, m, u = map(_arr, (Ahat, R, fbar, m, u))
         return self.L.ora_mpc_move_cost(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(fbar), _dp(m), _dp(u))
 
-    def mpc_bruteforce(self, Ahat, R, beta, lo, hi, m):
+    def mpc_bruteforce(self, Ahat, R, beta, lo, hi, m, dref=0.0, fbar=None):
         Ahat, R, lo, hi, m = map(_arr, (Ahat, R, lo, hi, m))
         u = np.zeros((self.M, self.n))
-        rc = self.L.ora_mpc_bruteforce(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(lo),
-                                       _dp(hi), _dp(m), _dp(u))
+        fb = _dp(_arr(fbar)) if fbar is not None else None
+        rc = self.L.ora_mpc_bruteforce_ref(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), float(dref), fb,
+                                           _dp(lo), _dp(hi), _dp(m), _dp(u))
         if rc != 0:
             raise ValueError("bruteforce needs M*N <= 10")
         return u
 
-    def mpc_cost(self, Ahat, R, beta, m, u):
+    def mpc_cost(self, Ahat, R, beta, m, u, dref=0.0):
         Ahat, R, m, u = map(_arr, (Ahat, R, m, u))
-        return self.L.ora_mpc_cost(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(m), _dp(u))
+        return self.L.ora_mpc_cost_ref(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), float(dref), _dp(m),
+                                       _dp(u))
 
-    def classify(self, Ahat, R, beta, lo, hi, m, u):
+    def ref_pow(self, i):
+        return self.L.ora_ref_pow(C.byref(self.cfg), int(i))
+
+    def classify(self, Ahat, R, beta, lo, hi, m, u, dref=0.0):
         Ahat, R, lo, hi, m, u = map(_arr, (Ahat, R, lo, hi, m, u))
         act = np.zeros(self.M, dtype=np.uint32); tie = np.zeros(self.M, dtype=np.uint32)
-        self.L.ora_mpc_classify(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), _dp(lo),
+        self.L.ora_mpc_classify_ref(C.byref(self.cfg), _dp(Ahat), _dp(R), float(beta), float(dref), _dp(lo),
                                 _dp(hi), _dp(m), _dp(u),
                                 act.ctypes.data_as(C.POINTER(C.c_uint32)),
                                 tie.ctypes.data_as(C.POINTER(C.c_uint32)))
