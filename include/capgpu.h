@@ -92,6 +92,10 @@ typedef struct {
                          >= 0 (W^2/MHz^2); 0 = the literal Eq. 9.  > 0 couples the M blocks: solved by a
                          generic per-instance active set, CUDA path for M * N <= 10, capgpu_simulate only
                          (not control_step / hierarchical / SLO schedule: CAPGPU_E_UNSUPPORTED) */
+  double ref_alpha;   /* NEXT-3 reference trajectory ("a reference trajectory"; Q37):
+                         prediction step i tracks r(k+i|k) = P_s - ref_alpha^i (P_s - p(k)) instead of
+                         P_s; ref_alpha = exp(-T/T_ref) in [0, 1), 0 = the literal Eq. 9 (r = P_s).
+                         Every call and config (also control_step / hierarchical / move / SLO). */
 } capgpu_params;
 
 /* Contiguous server range of this process (one process per GPU, §8(e)). */

@@ -40,7 +40,8 @@ class Params(C.Structure):
     _fields_ = [("q", C.c_double), ("r0", C.c_double), ("theta_min", C.c_double), ("lam", C.c_double),
                 ("rho", C.c_double), ("a_lo", C.c_double), ("a_hi", C.c_double), ("a_floor", C.c_double),
                 ("gamma", C.c_double), ("noise_std", C.c_double), ("substeps", C.c_int32),
-                ("caps_per_server", C.c_int32), ("seed", C.c_uint64), ("wmove", C.c_double)]
+                ("caps_per_server", C.c_int32), ("seed", C.c_uint64), ("wmove", C.c_double),
+                ("ref_alpha", C.c_double)]
 
 
 class Shard(C.Structure):
@@ -244,6 +245,7 @@ class CapGPU:
         p.gamma, p.noise_std, p.substeps = controller["gamma"], controller["noise_std"], controller["substeps"]
         p.caps_per_server, p.seed = caps_per_server, seed
         p.wmove = controller.get("wmove", 0.0)
+        p.ref_alpha = controller.get("ref_alpha", 0.0)
         sh = Shard()
         sh.rank, sh.world, sh.srv_begin = rank, world, srv_begin
         sh.n_servers_global = n_servers_global if n_servers_global is not None else srv_begin + n_servers

@@ -170,6 +170,8 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   if (!(prm.substeps == 1 || prm.substeps == 2 || prm.substeps == 4 || prm.substeps == 8))
     return fail(nullptr, CAPGPU_E_INVALID, "substeps must be 1, 2, 4 or 8");
   if (!(prm.wmove >= 0.0) || !std::isfinite(prm.wmove)) return fail(nullptr, CAPGPU_E_INVALID, "wmove must be >= 0");
+  if (!(prm.ref_alpha >= 0.0 && prm.ref_alpha < 1.0))
+    return fail(nullptr, CAPGPU_E_INVALID, "ref_alpha must be in [0, 1)");
   if (prm.wmove > 0.0 && h.M * N > kMoveMaxVars)
     return fail(nullptr, CAPGPU_E_UNSUPPORTED, "move suppression needs M * N <= %d on the CUDA path", kMoveMaxVars);
   for (int j = 0; j < N; ++j) {
@@ -226,6 +228,21 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   d.inv_S = 1.0 / (double)prm.substeps;
   d.inv_lam = 1.0 / prm.lambda;
   d.wmove = prm.wmove;
+  // Q37: block t's tracking offset is beta + ref_w[t] (P_s - p(k)), ref_w[t] =
+  // mean of alpha^i over the prediction steps i whose prediction uses u_t
+  d.ref = prm.ref_alpha > 0.0 ? 1 : 0;
+  for (int t = 0; t < h.M; ++t) {
+    double sum = 0.0, ai = 1.0;
+    int cnt = 0;
+    for (int i = 1; i <= h.P; ++i) {
+      ai *= prm.ref_alpha;
+      if ((i < h.M ? i : h.M) - 1 == t) {
+        sum += ai;
+        ++cnt;
+      }
+    }
+    d.ref_w[t] = d.ref ? sum / cnt : 0.0;
+  }
   // Q11: c_t = Q for t < M-1, c_{M-1} = (P - M + 1) Q
   for (int t = 0; t < h.M; ++t) d.ct[t] = t < h.M - 1 ? prm.q : (double)(h.P - h.M + 1) * prm.q;
   d.seed = prm.seed;

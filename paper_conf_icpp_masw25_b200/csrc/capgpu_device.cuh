@@ -92,6 +92,8 @@ struct DevParams {
   int32_t bl_kind, bl_steps;
   double bl_margin, bl_pole;
   double wmove;              // NEXT-3 move-suppression weight W (Q36); 0 = the literal Eq. 9
+  int32_t ref;               // NEXT-3 reference trajectory on (Q37): block t tracks beta + ref_w[t] (P_s - p(k))
+  double ref_w[kMaxM];
   int32_t no_chunking;       // 1: fused kernel without the chunked persistent schedule (env CAPGPU_NO_CHUNKING)
   long long *phase;          // [8][n_inst] cycle counters (builds with -DCAPGPU_PHASE_TIMING only)
   KnobConst k[kMaxN];
@@ -486,7 +488,7 @@ __device__ __forceinline__ uint32_t block_u(const KnobConst *kc, const double (&
 // branch-free and fully unrolled.  Half the Hessian (variable a = t N + j):
 //   H(a, a)  = c_t A_j^2 + R_j + W (1 + [t < M-1])
 //   H(a, b)  = c_t A_j A_k  (same t, k != j);  -W (same j, |t - t'| = 1)
-//   g(a)     = c_t beta A_j - R_j m_j - [t = 0] W f_j
+//   g(a)     = c_t beta_t A_j - R_j m_j - [t = 0] W f_j,  beta_t = beta + ref_w[t] dref (Q37)
 template <int N, int M>
 __device__ __forceinline__ double move_h(const DevParams &P, const double (&a)[N], const double (&R)[N], int x,
                                          int y) {
@@ -501,7 +503,7 @@ __device__ __forceinline__ double move_h(const DevParams &P, const double (&a)[N
 
 template <int N, int M>
 __device__ __forceinline__ uint32_t move_qp(const DevParams &P, const KnobConst *kc, const double (&a)[N],
-                                            const double (&R)[N], double beta, const double (&f)[N],
+                                            const double (&R)[N], double beta, double dref, const double (&f)[N],
                                             uint32_t (&act)[M], double (&x)[M * N]) {
   constexpr int V = M * N;
   double g[V];
@@ -511,7 +513,7 @@ __device__ __forceinline__ uint32_t move_qp(const DevParams &P, const KnobConst 
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       const int v = t * N + j;
-      g[v] = P.ct[t] * beta * a[j] - R[j] * kc[j].m - (t == 0 ? P.wmove * f[j] : 0.0);
+      g[v] = P.ct[t] * fma(P.ref_w[t], dref, beta) * a[j] - R[j] * kc[j].m - (t == 0 ? P.wmove * f[j] : 0.0);
       const uint32_t code = (act[t] >> (2 * j)) & 3u;
       lo_m |= (code == 1u ? 1u : 0u) << v;
       up_m |= (code == 2u ? 1u : 0u) << v;

@@ -405,7 +405,7 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
       smax = fma(ahat[j], P.k[j].hi, smax);
     }
     status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
-    status |= move_qp<N, M>(P, P.k, ahat, R, beta, fbar, act, u);
+    status |= move_qp<N, M>(P, P.k, ahat, R, beta, cap - p, fbar, act, u);
 #pragma unroll
     for (int j = 0; j < N; ++j) u0[j] = u[j];
 #pragma unroll
@@ -416,7 +416,7 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
     }
     return tsum * P.inv_N;
   }
-  if (P.convex) {
+  if (P.convex && !P.ref) {
     double smin = 0.0, smax = 0.0;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
@@ -522,7 +522,9 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
 #pragma unroll
     for (int j = 0; j < N; ++j) ctau[j] = c * tau[j];
     uint32_t code;
-    const double s = solve_block<N>(kc, kc_dev, ahat, ctau, beta, s_prev[0]);
+    // Q37: with the reference trajectory block t tracks beta + ref_w[t] (P_s - p(k))
+    const double beta_t = P.ref ? fma(P.ref_w[t], cap - p, beta) : beta;
+    const double s = solve_block<N>(kc, kc_dev, ahat, ctau, beta_t, s_prev[0]);
     code = block_codes<N>(kc, ctau, s);
     if (t == 0 || out.u) {
       double u[N];

@@ -25,8 +25,11 @@ def _desc(periods=K):
     return configs.get(4, periods=periods)
 
 
-def test_hierarchical_vs_oracle(G, oracle_mod):
+@pytest.mark.parametrize("ref_alpha", [0.0, 0.6])
+def test_hierarchical_vs_oracle(G, oracle_mod, ref_alpha):
+    """ref_alpha > 0: the NEXT-3 reference trajectory (Q37) on the per-period kernel."""
     d = _desc()
+    d["controller"]["ref_alpha"] = ref_alpha
     trs = np.array([0, 17, 1023, 1024, 2047])
     g = G.CapGPU.from_config(d, n_servers=N_SRV, n_servers_global=N_SRV)
     out = {k: H(v) for k, v in g.simulate(K, G.workload_from(d), trace_inst=trs).items()}
