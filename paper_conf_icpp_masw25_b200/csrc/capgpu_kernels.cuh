@@ -1195,12 +1195,12 @@ struct TileAcc {
 template <int N>
 struct PeriodTile {
   static constexpr int T = Tri<N>::size;
-  // Sigma | mu_f | Sfp | A0 | thr_max | base | amp; the read-only constants are
-  // staged only when the 128-thread tile fits the 227 KB of shared memory
-  // (N <= 15), else they are read from global memory where used.
-  static constexpr bool ro = (T + 6 * N) * kPeriodCta * 8 <= 227 * 1024;
+  // Sigma | mu_f | Sfp | A0 | thr_max | base | amp | a_true | C_true; the
+  // read-only constants are staged only when the tile fits the 227 KB of
+  // shared memory, else they are read from global memory where used.
+  static constexpr bool ro = (T + 7 * N + 1) * kPeriodCta * 8 <= 227 * 1024;
   static constexpr int oS = 0, oMU = T, oSFP = T + N, oA0 = T + 2 * N, oTM = T + 3 * N, oBA = T + 4 * N,
-                       oAM = T + 5 * N, F = ro ? T + 6 * N : T + 2 * N;
+                       oAM = T + 5 * N, oAT = T + 6 * N, oCT = T + 7 * N, F = ro ? T + 7 * N + 1 : T + 2 * N;
   static constexpr int bytes_per_cta = F * kPeriodCta * 8;
 };
 
@@ -1234,23 +1234,15 @@ __global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevPara
   const bool valid = i < P.n_srv;
   const int64_t ic = valid ? i : 0;
   const int64_t ld = P.n_srv;
-  // ---- S5: caps of instant k from the aggregates of instant k-1
-  const double w_prev = valid ? bd.srv_w[ic] : 0.0;
-  const double pmin_i = valid ? st.pmin[ic] : 0.0;
-  const double W = bd.agg[0];
-  const double Wr = group_sum(w_prev, bd.rack);
-  const double Pr = group_sum(pmin_i, bd.rack);
-  const double Bmax = bd.rack_frac * group_sum(valid ? st.pmax[ic] : 0.0, bd.rack);
-  const double Br = fmin(Bmax, fma(bd.B_c - bd.pmin_tot, Wr / W, Pr));
-  const double cap = fma(Br - Pr, w_prev / Wr, pmin_i);
-  double tbar = 0.0, p = 0.0;
   using PT = PeriodTile<N>;
   extern __shared__ __align__(16) double ptile[];
   double *tile = ptile + (threadIdx.x >> 5) * (PT::F * 32) + (threadIdx.x & 31);
+  // Every load of the period is issued in one batch before anything waits:
+  // the model state and read-only constants into this warp's tile
+  // (asynchronous, no registers held), the rest into registers.  (One memory
+  // round trip per server and period; dependent loads issued later would each
+  // add a DRAM latency to the period.)
   if (valid) {
-    // Stage Sigma, mu_f, Sfp and the read-only constants into this warp's tile
-    // (asynchronous, no registers held), load what crosses the period (fbar,
-    // acc, thr) into registers, then wait once.
 #pragma unroll
     for (int t = 0; t < PT::T; ++t) cp_async8(tile + (PT::oS + t) * 32, st.S + t * ld + i);
 #pragma unroll
@@ -1262,30 +1254,51 @@ __global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevPara
         cp_async8(tile + (PT::oTM + j) * 32, st.thr_max + j * ld + i);
         cp_async8(tile + (PT::oBA + j) * 32, st.base + j * ld + i);
         cp_async8(tile + (PT::oAM + j) * 32, st.amp + j * ld + i);
+        cp_async8(tile + (PT::oAT + j) * 32, st.a_true + j * ld + i);
       }
     }
-    double fbar[N], acc[N], thr[N];
+    if constexpr (PT::ro) cp_async8(tile + PT::oCT * 32, st.c_true + i);
+  }
+  double fbar[N], acc[N], thr[N], s_prev[M];
+  uint32_t act[M];
+  double w = 0.0, mu_p = 0.0, p = 0.0;
+  int slot = -1;
+  if (valid) {
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       fbar[j] = st.fbar[j * ld + i];
       acc[j] = st.acc[j * ld + i];
       thr[j] = st.thr[j * ld + i];
     }
-    cp_async_wait_all();
-    const TileAcc S{tile + PT::oS * 32}, MUF{tile + PT::oMU * 32}, SFP{tile + PT::oSFP * 32};
-    using RO = PeriodRo<PT::ro>;
-    const typename RO::type A0a = RO::make(tile, PT::oA0, st.A0, i, ld), TMa = RO::make(tile, PT::oTM, st.thr_max, i, ld),
-                            BAa = RO::make(tile, PT::oBA, st.base, i, ld), AMa = RO::make(tile, PT::oAM, st.amp, i, ld);
-    double w = st.w[i], mu_p = st.mu_p[i];
+    w = st.w[i];
+    mu_p = st.mu_p[i];
     p = st.p[i];
-    double s_prev[M];
-    uint32_t act[M], status;
 #pragma unroll
     for (int t = 0; t < M; ++t) {
       s_prev[t] = st.s_prev[t * ld + i];
       act[t] = st.act[t * ld + i];
     }
-    const int slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
+    slot = tr.n_trace > 0 ? st.trace_slot[i] : -1;
+  }
+  // ---- S5: caps of instant k from the aggregates of instant k-1
+  const double w_prev = valid ? bd.srv_w[ic] : 0.0;
+  const double pmin_i = valid ? st.pmin[ic] : 0.0;
+  const double pmax_i = valid ? st.pmax[ic] : 0.0;
+  const double W = bd.agg[0];
+  const double Wr = group_sum(w_prev, bd.rack);
+  const double Pr = group_sum(pmin_i, bd.rack);
+  const double Bmax = bd.rack_frac * group_sum(pmax_i, bd.rack);
+  const double Br = fmin(Bmax, fma(bd.B_c - bd.pmin_tot, Wr / W, Pr));
+  const double cap = fma(Br - Pr, w_prev / Wr, pmin_i);
+  double tbar = 0.0;  // p stays p(k): the CTA partial below sums the instant-k powers
+  if (valid) {
+    cp_async_wait_all();
+    const TileAcc S{tile + PT::oS * 32}, MUF{tile + PT::oMU * 32}, SFP{tile + PT::oSFP * 32};
+    using RO = PeriodRo<PT::ro>;
+    const typename RO::type A0a = RO::make(tile, PT::oA0, st.A0, i, ld), TMa = RO::make(tile, PT::oTM, st.thr_max, i, ld),
+                            BAa = RO::make(tile, PT::oBA, st.base, i, ld), AMa = RO::make(tile, PT::oAM, st.amp, i, ld),
+                            ATa = RO::make(tile, PT::oAT, st.a_true, i, ld);
+    uint32_t status;
     InstantOut io{};
     if (slot >= 0) {
       io.ld = tr.n_trace;
@@ -1306,6 +1319,25 @@ __global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevPara
       if (tr.active) {
 #pragma unroll
         for (int t = 0; t < M; ++t) tr.active[((int64_t)kk * M + t) * tr.n_trace + slot] = act[t];
+      }
+    }
+    // the running summaries (read-modify-write over the window, Q25) are
+    // loaded here so their latency overlaps the plant instead of following it
+    const int kw = K - (4 * K) / 5;
+    const bool win = kk >= kw, first = kk == kw;
+    double o_sum = 0.0, o_sq = 0.0, o_max = 0.0, o_th = 0.0;
+    int o_viol = 0, o_ac[M];
+#pragma unroll
+    for (int t = 0; t < M; ++t) o_ac[t] = 0;
+    if (win && !first) {
+      if (tr.sum_p) o_sum = tr.sum_p[i];
+      if (tr.sumsq_p) o_sq = tr.sumsq_p[i];
+      if (tr.max_p) o_max = tr.max_p[i];
+      if (tr.sum_theta) o_th = tr.sum_theta[i];
+      if (tr.n_viol) o_viol = tr.n_viol[i];
+      if (tr.act_count) {
+#pragma unroll
+        for (int t = 0; t < M; ++t) o_ac[t] = tr.act_count[t * ld + i];
       }
     }
     // ---- S4: period k -> k+1
@@ -1330,24 +1362,22 @@ __global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevPara
     else
       plant_delta_sigma<N>(P, P.grid, u0, acc, dem, thr_max, fbar, thr);
     const double noise = gen_noise(gen_stream_key(P.seed, GEN_TAG_NOISE, srv), k + 1, P.noise_scale);
-    double pw = st.c_true[i];
+    double pw = PT::ro ? tile[PT::oCT * 32] : st.c_true[i];
 #pragma unroll
-    for (int j = 0; j < N; ++j) pw = fma(st.a_true[j * ld + i], fbar[j], pw);
+    for (int j = 0; j < N; ++j) pw = fma(ATa.get(j), fbar[j], pw);
     const double p_next = pw + noise;
     // ---- summaries over the last 80 % of the call's periods (Q25)
-    const int kw = K - (4 * K) / 5;
-    if (kk >= kw) {
-      const bool first = kk == kw;
-      if (tr.sum_p) tr.sum_p[i] = (first ? 0.0 : tr.sum_p[i]) + p_next;
-      if (tr.sumsq_p) tr.sumsq_p[i] = fma(p_next, p_next, first ? 0.0 : tr.sumsq_p[i]);
-      if (tr.max_p) tr.max_p[i] = first ? p_next : fmax(tr.max_p[i], p_next);
-      if (tr.sum_theta) tr.sum_theta[i] = (first ? 0.0 : tr.sum_theta[i]) + tbar;
-      if (tr.n_viol) tr.n_viol[i] = (first ? 0 : tr.n_viol[i]) + (p_next > cap ? 1 : 0);
+    if (win) {
+      if (tr.sum_p) tr.sum_p[i] = o_sum + p_next;
+      if (tr.sumsq_p) tr.sumsq_p[i] = fma(p_next, p_next, o_sq);
+      if (tr.max_p) tr.max_p[i] = first ? p_next : fmax(o_max, p_next);
+      if (tr.sum_theta) tr.sum_theta[i] = o_th + tbar;
+      if (tr.n_viol) tr.n_viol[i] = o_viol + (p_next > cap ? 1 : 0);
       if (tr.n_window) tr.n_window[i] = K - kw;
       if (tr.n_miss && first) tr.n_miss[i] = 0;  // no SLO schedule with the budget
       if (tr.act_count) {
 #pragma unroll
-        for (int t = 0; t < M; ++t) tr.act_count[t * ld + i] = (first ? 0 : tr.act_count[t * ld + i]) + (act[t] != 0u);
+        for (int t = 0; t < M; ++t) tr.act_count[t * ld + i] = o_ac[t] + (act[t] != 0u);
       }
     }
     if (tr.final_p && kk == K - 1) tr.final_p[i] = p_next;
