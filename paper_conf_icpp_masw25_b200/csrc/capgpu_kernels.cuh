@@ -1173,11 +1173,12 @@ __device__ __forceinline__ void cta_sum2(double a, double b, double *out_a, doub
 }
 
 // Servers per CTA of the per-period kernel (and of the S5 CTA partial sums:
-// 1024-server budget blocks are kBudgetBlock / kPeriodCta CTAs).  64: four
-// CTAs per SM (register and shared-memory limits at N = 9), so the stage-in,
-// compute and write-back phases of different CTAs overlap.
+// 1024-server budget blocks are kBudgetBlock / kPeriodCta CTAs).  32: eight
+// one-warp CTAs per SM (register and shared-memory limits at N = 9), so the
+// stage-in, compute and write-back phases of different CTAs overlap (64: four
+// two-warp CTAs, measured the same within noise).
 #ifndef CAPGPU_PERIOD_CTA
-#define CAPGPU_PERIOD_CTA 64
+#define CAPGPU_PERIOD_CTA 32
 #endif
 constexpr int kPeriodCta = CAPGPU_PERIOD_CTA;
 
@@ -1225,43 +1226,46 @@ __device__ __forceinline__ void cp_async8(double *smem_dst, const double *gsrc) 
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
-// One instant of the hierarchical configuration for every local server:
-// budget caps, S1-S3, the w_i / p partial sums, S4.  State in HBM.
+// cp.async of the server's model state and read-only constants into its tile
+// column (tile = warp tile base + lane)
+template <int N>
+__device__ __forceinline__ void period_stage(const StatePtrs &st, int64_t i, int64_t ld, double *tile) {
+  using PT = PeriodTile<N>;
+#pragma unroll
+  for (int t = 0; t < PT::T; ++t) cp_async8(tile + (PT::oS + t) * 32, st.S + t * ld + i);
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    cp_async8(tile + (PT::oMU + j) * 32, st.mu_f + j * ld + i);
+    cp_async8(tile + (PT::oSFP + j) * 32, st.Sfp + j * ld + i);
+    if constexpr (PT::ro) {
+      cp_async8(tile + (PT::oA0 + j) * 32, st.A0 + j * ld + i);
+      cp_async8(tile + (PT::oTM + j) * 32, st.thr_max + j * ld + i);
+      cp_async8(tile + (PT::oBA + j) * 32, st.base + j * ld + i);
+      cp_async8(tile + (PT::oAM + j) * 32, st.amp + j * ld + i);
+      cp_async8(tile + (PT::oAT + j) * 32, st.a_true + j * ld + i);
+    }
+  }
+  if constexpr (PT::ro) cp_async8(tile + PT::oCT * 32, st.c_true + i);
+}
+
+
+// One server of one instant (everything after the tile's cp.async was
+// issued): the register loads, S5 caps, S1-S4, summaries and write-back.
+// Returns tbar (w_i) and leaves p = p(k) for the CTA partials.  (A
+// double-buffered persistent variant -- next tile's cp.async in flight while
+// computing -- was measured slower: 4 resident warps per SM, 1.38 vs 1.92 G
+// steps/s at cfg 4; the compute phase needs the 8 warps.)
 template <int N, int M, int SS>
-__global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
-                                                int kk, int K) {
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const bool valid = i < P.n_srv;
+__device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs &st, const BudgetDev &bd,
+                                            const TracePtrs &tr, int64_t k, int kk, int K, int64_t i, bool valid,
+                                            double *tile, double &tbar, double &p) {
   const int64_t ic = valid ? i : 0;
   const int64_t ld = P.n_srv;
   using PT = PeriodTile<N>;
-  extern __shared__ __align__(16) double ptile[];
-  double *tile = ptile + (threadIdx.x >> 5) * (PT::F * 32) + (threadIdx.x & 31);
-  // Every load of the period is issued in one batch before anything waits:
-  // the model state and read-only constants into this warp's tile
-  // (asynchronous, no registers held), the rest into registers.  (One memory
-  // round trip per server and period; dependent loads issued later would each
-  // add a DRAM latency to the period.)
-  if (valid) {
-#pragma unroll
-    for (int t = 0; t < PT::T; ++t) cp_async8(tile + (PT::oS + t) * 32, st.S + t * ld + i);
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-      cp_async8(tile + (PT::oMU + j) * 32, st.mu_f + j * ld + i);
-      cp_async8(tile + (PT::oSFP + j) * 32, st.Sfp + j * ld + i);
-      if constexpr (PT::ro) {
-        cp_async8(tile + (PT::oA0 + j) * 32, st.A0 + j * ld + i);
-        cp_async8(tile + (PT::oTM + j) * 32, st.thr_max + j * ld + i);
-        cp_async8(tile + (PT::oBA + j) * 32, st.base + j * ld + i);
-        cp_async8(tile + (PT::oAM + j) * 32, st.amp + j * ld + i);
-        cp_async8(tile + (PT::oAT + j) * 32, st.a_true + j * ld + i);
-      }
-    }
-    if constexpr (PT::ro) cp_async8(tile + PT::oCT * 32, st.c_true + i);
-  }
   double fbar[N], acc[N], thr[N], s_prev[M];
   uint32_t act[M];
-  double w = 0.0, mu_p = 0.0, p = 0.0;
+  double w = 0.0, mu_p = 0.0;
+  p = 0.0;
   int slot = -1;
   if (valid) {
 #pragma unroll
@@ -1290,7 +1294,7 @@ __global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevPara
   const double Bmax = bd.rack_frac * group_sum(pmax_i, bd.rack);
   const double Br = fmin(Bmax, fma(bd.B_c - bd.pmin_tot, Wr / W, Pr));
   const double cap = fma(Br - Pr, w_prev / Wr, pmin_i);
-  double tbar = 0.0;  // p stays p(k): the CTA partial below sums the instant-k powers
+  tbar = 0.0;  // p stays p(k): the CTA partial sums the instant-k powers
   if (valid) {
     cp_async_wait_all();
     const TileAcc S{tile + PT::oS * 32}, MUF{tile + PT::oMU * 32}, SFP{tile + PT::oSFP * 32};
@@ -1402,6 +1406,25 @@ __global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevPara
     }
     bd.srv_w[i] = tbar;
   }
+}
+
+// One instant of the hierarchical configuration for every local server:
+// budget caps, S1-S3, the w_i / p partial sums, S4.  State in HBM.
+template <int N, int M, int SS>
+__global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
+                                                int kk, int K) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const bool valid = i < P.n_srv;
+  using PT = PeriodTile<N>;
+  extern __shared__ __align__(16) double ptile[];
+  double *tile = ptile + (threadIdx.x >> 5) * (PT::F * 32) + (threadIdx.x & 31);
+  // Every load of the period is issued in one batch before anything waits:
+  // the model state and read-only constants into this warp's tile
+  // (asynchronous, no registers held), the rest into registers (one memory
+  // round trip per server and period).
+  if (valid) period_stage<N>(st, i, P.n_srv, tile);
+  double tbar, p;
+  period_body<N, M, SS>(P, st, bd, tr, k, kk, K, i, valid, tile, tbar, p);
   const int n_cta = gridDim.x;
   cta_sum2<kPeriodCta>(tbar, p, &bd.cta_part[blockIdx.x], &bd.cta_part[n_cta + blockIdx.x]);
 }
