@@ -54,6 +54,8 @@ def _deps():
 VARIANTS = {
     # profiling build: per-phase cycle counters in the fused kernel (never the product library)
     "timing": (["-DCAPGPU_PHASE_TIMING"], "_build_timing", "libcapgpu_timing.so"),
+    # A/B experiments: the working tree built beside the product library
+    "exp": ([], "_build_exp", "libcapgpu_exp.so"),
 }
 
 
