@@ -131,7 +131,17 @@ def _oracle_worker(args):
     return time.perf_counter() - t
 
 
-def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int):
+def cpu_model() -> str:
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int, single: dict | None = None):
     """Oracle (as it stands) on `cores` host processes over a bounded sample of
     the workload; returns (steps/s, sample description, cores)."""
     import multiprocessing as mp
@@ -141,8 +151,11 @@ def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int):
     n_inst = desc["n_servers"] * desc["workload"]["n_caps"]
     cal_p = min(periods, 100)
     t_cal = _oracle_worker((desc, [0], cal_p))
+    if single is not None:  # the single-core rate beside the all-cores one
+        single["single_core"] = cal_p / t_cal
     per_inst = t_cal / cal_p * periods
     k = max(1, int(budget_s / max(per_inst, 1e-6)))
+    k = min(k, max(1, -(-n_inst // cores)))  # never more than the whole workload
     stride = max(1, n_inst // (k * cores))
     jobs = [(desc, [((w * k + i) * stride) % n_inst for i in range(k)], periods) for w in range(cores)]
     ctx = mp.get_context("fork")
@@ -189,7 +202,8 @@ def run_reference(args):
     total_steps, total_t = 0.0, 0.0
     budget = max(1.0, 60.0 / max(1, args.steps + args.warmup))
     for it in range(args.warmup + args.steps):
-        rate, sample, cores_used, wall = oracle_rate(args.config, periods, budget, cores)
+        extra = {}
+        rate, sample, cores_used, wall = oracle_rate(args.config, periods, budget, cores, extra)
         if it >= args.warmup:
             total_steps += rate * wall
             total_t += wall
@@ -201,7 +215,8 @@ def run_reference(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded, DESIGN.md §3)",
             "config": {"workload": workload_name(d, periods), "n_knobs": N, "P": d["P"], "M": d["M"]},
             "cpu_baseline": {"value": value, "unit": "server-control-steps/s", "cores": cores_used,
-                             "kind": "oracle", "sample": sample},
+                             "kind": "oracle", "sample": sample, "cpu_model": cpu_model(),
+                             "single_core": extra.get("single_core")},
             "e2e": {"value": value, "unit": "server-control-steps/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -380,9 +395,11 @@ def main():
                 "gpu_launches": launches,
                 "clocks": clocks}
         if world == 1 and not args.no_cpu_baseline:
-            rate, sample, cores, _ = oracle_rate(args.config, periods, args.cpu_budget, os.cpu_count() or 1)
+            extra = {}
+            rate, sample, cores, _ = oracle_rate(args.config, periods, args.cpu_budget, os.cpu_count() or 1, extra)
             line["cpu_baseline"] = {"value": rate, "unit": "server-control-steps/s", "cores": cores,
-                                    "kind": "oracle", "sample": sample}
+                                    "kind": "oracle", "sample": sample, "cpu_model": cpu_model(),
+                                    "single_core": extra.get("single_core")}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
