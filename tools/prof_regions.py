@@ -26,8 +26,9 @@ for f, p in SRC.items():
         if m:
             st.append((i, m.group(1)))
     starts[f] = st
-sass = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
-                      capture_output=True, text=True).stdout
+sass = (open(rep).read() if rep.endswith(".csv") else
+        subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                       capture_output=True, text=True).stdout)
 srows = list(csv.reader(io.StringIO(sass)))
 sh, sd = srows[1], srows[2:]
 tmp = tempfile.mkdtemp()
