@@ -391,7 +391,9 @@ def main():
                 "roofline": roof,
                 "e2e": {"value": e2e_value, "unit": "server-control-steps/s",
                         "h2d_bytes_per_step": 0 if hier else 8 * n_inst,
-                        "d2h_bytes_per_step": 20 * n_inst},
+                        "d2h_bytes_per_step": 20 * n_inst,
+                        **({"note": "no per-step host inputs: the hierarchical caps are computed on the "
+                                    "device from the cluster budget every period (Q16)"} if hier else {})},
                 "gpu_launches": launches,
                 "clocks": clocks}
         if world == 1 and not args.no_cpu_baseline:
