@@ -1688,15 +1688,20 @@ int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int
   const int64_t n_groups = (P.n_inst + BLOCK - 1) / BLOCK;
   if constexpr (can_chunk) {
     auto kc = k_simulate<N, M, S, BLOCK, false, false, true>;
-    int occ = 0, dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kc, BLOCK, smem) != cudaSuccess) {
-      cudaGetLastError();
-      occ = 0;
+    // resident slots of the chunked instantiation (probed once per process;
+    // one device per process, §8(e))
+    static int64_t slots = -1;
+    if (slots < 0) {
+      int occ = 0, dev = 0, sms = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      if (cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kc, BLOCK, smem) != cudaSuccess) {
+        cudaGetLastError();
+        occ = 0;
+      }
+      slots = (int64_t)occ * sms;
     }
-    const int64_t slots = (int64_t)occ * sms;
     C = (st.sched && slots > 0 && !P.no_chunking) ? sim_chunks(n_groups, slots, K) : 1;
     if (C > 1) {
       SimSched sc{};
@@ -1707,6 +1712,7 @@ int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int
       sc.n_items = (int32_t)(n_groups * ((K + sc.Kc - 1) / sc.Kc));
       cudaError_t e = cudaMemsetAsync(st.sched, 0, sizeof(int32_t) * (size_t)(P.n_inst + 1), s);
       if (e != cudaSuccess) return (int)e;
+      cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       kc<<<(unsigned)sc.n_items, BLOCK, smem, s>>>(P, st, tr, k0, K, sc);
       return (int)cudaGetLastError();
     }
