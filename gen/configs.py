@@ -24,10 +24,10 @@ _BASE_WORKLOAD = dict(n_caps=1, demand_kind=1, demand_frac=0.7, cap_frac0=0.5, c
                       cap_frac_step=0.0, cap_period=0, cap_lo=0, cap_hi=0, cap_mult=1.0,
                       hierarchical=False, gain_dlo=0.0, gain_step=0.0,
                       slo_period=0, slo_lo=0, slo_hi=0, slo_a=None, slo_b=None,
-                      controller=0, fs_levels=1, safe_margin=0.0, p_pole=0.5)
+                      controller=0, fs_levels=1, safe_margin=0.0, p_pole=0.5, gpu_share=0.5)
 
 # NEXT-2 baseline controllers (§6.1): workload["controller"]
-CONTROLLERS = {"capgpu": 0, "fixed": 1, "safe": 2, "gpuonly": 3, "cpuonly": 4}
+CONTROLLERS = {"capgpu": 0, "fixed": 1, "safe": 2, "gpuonly": 3, "cpuonly": 4, "cpugpu": 5}
 
 # NEXT-1 (§6.4): latency SLOs as ratios SLO_j / e_min,j for the three
 # tail levels the paper switches between ("30 %", "50 %", "80 % tail").  The
@@ -97,17 +97,19 @@ def slo_schedule(n_servers: int = 64, periods: int = 1000, slo_period: int = 200
 
 
 def baseline(controller: str, n_servers: int = 1024, periods: int = 1000, fs_levels: int = 1,
-             safe_margin: float = 25.0, p_pole: float = 0.5, slo: bool = False) -> dict:
+             safe_margin: float = 25.0, p_pole: float = 0.5, slo: bool = False, gpu_share: float = 0.5) -> dict:
     """NEXT-2: a comparison controller (§6.1) on the cfg 2 plant and
     set-point schedule (1 CPU + 4 GPUs, P_min + 0.45 dP, x 900/800 in [40, 80)
     mod 200: the Fig. 10 step).  "fixed" / "safe" = Fixed-step /
     Safe Fixed-step (step `fs_levels` grid levels; safe set point
     P_s - safe_margin), "gpuonly" / "cpuonly" = pole-placed P loops
-    (pole p_pole), "capgpu" = the MPC on the same workload.
+    (pole p_pole), "cpugpu" = CPU+GPU, two such loops on separately
+    metered CPU and GPU power with the budget split gpu_share : 1 - gpu_share
+    (50/50 and 60/40; Q39), "capgpu" = the MPC on the same workload.
     slo=True adds the §6.4 SLO schedule (the baselines ignore it; misses count)."""
     d = get(2, n_servers=n_servers, periods=periods)
     d["workload"].update(controller=CONTROLLERS[controller], fs_levels=fs_levels, safe_margin=safe_margin,
-                         p_pole=p_pole)
+                         p_pole=p_pole, gpu_share=gpu_share)
     if slo:
         d["workload"].update(slo_period=200, slo_lo=14, slo_hi=114, slo_a=[0.0] + [SLO_TAIL[50]] * 4,
                              slo_b=[0.0, SLO_TAIL[30], SLO_TAIL[80], SLO_TAIL[80], SLO_TAIL[80]])

@@ -66,12 +66,18 @@ typedef struct {
   int64_t slo_period, slo_lo, slo_hi;
   double slo_a[ORA_MAXN], slo_b[ORA_MAXN];
   /* Baseline controllers (NEXT-2, §6.1; Q32-Q35) replacing S1-S3:
-   * 0 = CapGPU (MPC), 1 = Fixed-step, 2 = Safe Fixed-step, 3 = GPU-only, 4 = CPU-only. */
+   * 0 = CapGPU (MPC), 1 = Fixed-step, 2 = Safe Fixed-step, 3 = GPU-only, 4 = CPU-only,
+   * 5 = CPU+GPU (two loops on separately metered CPU and GPU power; Q39). */
   int32_t controller;
   int32_t fs_levels;   /* Fixed-step size in grid levels (stepsize 1 or 5) */
   double safe_margin;  /* Safe Fixed-step: set point lowered by this many W */
   double p_pole;       /* GPU-/CPU-only: closed-loop pole z of the pole-placed P gain */
+  double gpu_share;    /* CPU+GPU: GPU share of the server budget (50 % or 60 %) */
 } ora_workload;
+
+/* CPU+GPU (Q39): the CPU meter reads ORA_CPU_IDLE_SHARE * C + a_0 fbar_0 + n / 2,
+ * the GPU meter the rest of the server power. */
+#define ORA_CPU_IDLE_SHARE 0.3
 
 /* per-instance summary over the last 80 % of periods */
 typedef struct {

@@ -59,7 +59,7 @@ class OraWorkload(C.Structure):
                 ("slo_period", C.c_int64), ("slo_lo", C.c_int64), ("slo_hi", C.c_int64),
                 ("slo_a", C.c_double * MAXN), ("slo_b", C.c_double * MAXN),
                 ("controller", C.c_int32), ("fs_levels", C.c_int32), ("safe_margin", C.c_double),
-                ("p_pole", C.c_double)]
+                ("p_pole", C.c_double), ("gpu_share", C.c_double)]
 
 
 class OraSummary(C.Structure):
@@ -190,6 +190,7 @@ def make_workload(desc: dict, periods: int | None = None) -> OraWorkload:
         w.slo_b[j] = r
     w.controller, w.fs_levels = wl.get("controller", 0), wl.get("fs_levels", 1)
     w.safe_margin, w.p_pole = wl.get("safe_margin", 0.0), wl.get("p_pole", 0.5)
+    w.gpu_share = wl.get("gpu_share", 0.5)
     return w
 
 
@@ -421,7 +422,7 @@ class Oracle:
         return out
 
     def simulate_baseline(self, inst, periods=None, traces=True):
-        """NEXT-2 baseline controller of the workload (controller 1..4) on the same plant."""
+        """NEXT-2 baseline controller of the workload (controller 1..5) on the same plant."""
         inst = np.ascontiguousarray(np.asarray(inst, dtype=np.int64))
         ni = len(inst)
         w = make_workload(self.desc, periods)

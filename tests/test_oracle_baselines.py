@@ -129,3 +129,57 @@ def test_baselines_ignore_slo_but_misses_are_counted(oracle_mod):
     cg = oracle_mod.Oracle(configs.baseline("capgpu", n_servers=n, periods=K, slo=True))
     m = cg.simulate(range(n), traces=False)["summary"]["n_miss"]
     assert m.sum() == 0 and b.sum() > 0
+
+
+@pytest.mark.parametrize("share,z", [(0.82, 0.5), (0.8, 0.0), (0.83, 0.7)])
+def test_cpu_gpu_two_loops(oracle_mod, share, z):
+    """CPU+GPU (Q39): the CPU loop tracks (1 - share) P_s on the CPU
+    meter, the GPU loop share * P_s on the GPU meter, each with its own
+    pole-placed gain.  The meters are recomputed here from the traced level
+    indices with the grid formula and the TRUE gains (CPU meter
+    0.3 C + a_0 fbar_0 without noise); each loop's error obeys
+    |e(k+1) - z e(k)| <= sum_J a_j 2 step_j / S on unsaturated periods."""
+    d = _quiet("cpugpu", p_pole=z, periods=200, gpu_share=share)
+    o = oracle_mod.Oracle(d)
+    out = o.simulate_baseline(range(6))
+    N, S = o.n, d["controller"]["substeps"]
+    grid = _grid(d)
+    steps = np.array([(k["f_max"] - k["f_min"]) / (k["n_levels"] - 1) for k in d["knobs"]])
+    fmin = np.array([k["f_min"] for k in d["knobs"]]); fmax = np.array([k["f_max"] for k in d["knobs"]])
+    for i in range(6):
+        g = o.gen_server(i)
+        a, c0 = g["a_true"], g["c_true"]
+        u, p, cap, lv = out["u"][:, i], out["p"][:, i], out["cap"][:, i], out["levels"][:, i]
+        assert np.all(u[:, 1:] == u[:, [1]])  # one common GPU frequency
+        # fbar(k+1) from the levels applied in period k (grid formula, not the oracle's tables)
+        fb0 = np.array([np.mean(grid[0][lv[k, :, 0]]) for k in range(len(p))])
+        pc = 0.3 * c0 + a[0] * fb0[:-1]          # CPU meter at instants 1..K-1
+        pg = p[1:] - pc                           # GPU meter
+        ec = (1 - share) * cap[1:] - pc
+        eg = share * cap[1:] - pg
+        bc = a[0] * 2 * steps[0] / S + 1e-9
+        bg = np.sum(a[1:] * 2 * steps[1:] / S) + 1e-9
+        n_c = n_g = 0
+        for k in range(2, len(ec) - 1):
+            if fmin[0] < u[k + 1, 0] < fmax[0] and fmin[0] < u[k, 0] < fmax[0]:
+                assert abs(ec[k + 1] - z * ec[k]) <= bc, (i, k, ec[k + 1], z * ec[k])
+                n_c += 1
+            if fmin[1] < u[k + 1, 1] < fmax[1] and fmin[1] < u[k, 1] < fmax[1]:
+                assert abs(eg[k + 1] - z * eg[k]) <= bg, (i, k, eg[k + 1], z * eg[k])
+                n_g += 1
+        assert n_c + n_g > 100
+
+
+def test_cpu_gpu_fixed_split_misses_the_cap(oracle_mod):
+    """P:282 "it is hard to find the perfect ratio": the paper's 50/50 split
+    asks the CPU for more than it can draw (CPU meter 150-265 W of a ~1 kW
+    cap), the CPU saturates at f_max and the server settles below the cap; a
+    95 % GPU share pins the CPU at f_min and the GPU loop drives the server
+    over the cap."""
+    for share, cpu_pin, sign in [(0.5, "f_max", -1.0), (0.95, "f_min", 1.0)]:
+        d = _quiet("cpugpu", periods=200, gpu_share=share)
+        out = oracle_mod.Oracle(d).simulate_baseline(range(6))
+        assert np.all(out["u"][50:, :, 0] == d["knobs"][0][cpu_pin])
+        s = out["summary"]
+        dev = s["sum_p"] / s["n_window"] - out["cap"][-1]
+        assert np.all(sign * dev > 5.0), (share, dev)
