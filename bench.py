@@ -174,7 +174,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo", "fixed", "safe", "gpuonly", "cpuonly", "move"])
+    ap.add_argument("--config", default="3", choices=["1", "2", "3", "4", "5", "stab", "slo", "fixed", "safe", "gpuonly", "cpuonly", "cpugpu", "move"])
     ap.add_argument("--periods", type=int, default=None, help="control periods per bench step")
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")

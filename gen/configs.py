@@ -134,7 +134,7 @@ def by_name(name) -> dict:
     """bench.py --config: "1".."5" (BASELINE.json configs), "stab" (the NEXT-4
     gain sweep at bench size: 16,384 servers x 24 gains x 1,000 periods) or
     "slo" (the NEXT-1 SLO schedule: 1,048,576 servers x 1,000 periods), or a
-    NEXT-2 baseline "fixed" / "safe" / "gpuonly" / "cpuonly" (1,048,576 servers
+    NEXT-2 baseline "fixed" / "safe" / "gpuonly" / "cpuonly" / "cpugpu" (1,048,576 servers
     of the cfg 2 plant x 1,000 periods)."""
     if str(name) == "stab":
         return stability_sweep(n_servers=16384)

@@ -140,7 +140,10 @@ typedef struct {
    * with the highest (p < P_s) or lowest (p > P_s) theta by fs_levels grid levels
    * (ties round-robin; Safe Fixed-step uses P_s - safe_margin); GPU-only / CPU-only
    * run g(k) = clamp(g(k-1) + K (P_s - p(k))) on one common GPU (CPU) frequency
-   * with the other knobs at f_max and the pole-placed gain K = (1 - p_pole) / sum_J A0_j.
+   * with the other knobs at f_max and the pole-placed gain K = (1 - p_pole) / sum_J A0_j;
+   * CPU+GPU (Q39) runs one such loop per device class on its own meter (CPU
+   * meter 0.3 C + a_0 fbar_0 + n/2, GPU meter the rest) toward gpu_share * P_s (GPUs)
+   * and (1 - gpu_share) * P_s (CPU).
    * Traces: u row 0 = the command, theta, p, cap, levels; status 0; act_count 0.
    * The controller is fixed for a simulation (first call after create/sim_reset).
    * Not supported with `hierarchical`. */
@@ -148,10 +151,11 @@ typedef struct {
   int32_t fs_levels;   /* >= 1 */
   double safe_margin;  /* W, finite */
   double p_pole;       /* in [0, 1) */
+  double gpu_share;    /* CPU+GPU: GPU share of the budget, in (0, 1) */
 } capgpu_workload;
 
 enum { CAPGPU_CTRL_CAPGPU = 0, CAPGPU_CTRL_FIXED_STEP = 1, CAPGPU_CTRL_SAFE_FIXED_STEP = 2,
-       CAPGPU_CTRL_GPU_ONLY = 3, CAPGPU_CTRL_CPU_ONLY = 4 };
+       CAPGPU_CTRL_GPU_ONLY = 3, CAPGPU_CTRL_CPU_ONLY = 4, CAPGPU_CTRL_CPU_GPU = 5 };
 
 /* Optional outputs of capgpu_simulate; every pointer may be NULL.
  * Summaries are over the last floor(0.8 K) of the K periods of the call (Q25).

@@ -59,7 +59,7 @@ class Workload(C.Structure):
                 ("slo_period", C.c_int64), ("slo_lo", C.c_int64), ("slo_hi", C.c_int64),
                 ("slo_a", C.c_double * MAX_KNOBS), ("slo_b", C.c_double * MAX_KNOBS),
                 ("controller", C.c_int32), ("fs_levels", C.c_int32), ("safe_margin", C.c_double),
-                ("p_pole", C.c_double)]
+                ("p_pole", C.c_double), ("gpu_share", C.c_double)]
 
 
 _VP = C.c_void_p
@@ -218,6 +218,7 @@ def workload_from(desc: dict) -> Workload:
         w.slo_b[j] = r
     w.controller, w.fs_levels = wl.get("controller", 0), wl.get("fs_levels", 1)
     w.safe_margin, w.p_pole = wl.get("safe_margin", 0.0), wl.get("p_pole", 0.5)
+    w.gpu_share = wl.get("gpu_share", 0.5)
     return w
 
 

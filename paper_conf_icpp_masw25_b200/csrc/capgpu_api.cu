@@ -582,6 +582,7 @@ static void apply_workload(DevParams &d, const capgpu_workload &w) {
   d.bl_steps = w.fs_levels;
   d.bl_margin = w.safe_margin;
   d.bl_pole = w.p_pole;
+  d.bl_share = w.gpu_share;
 }
 
 }  // extern "C"
@@ -601,12 +602,14 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
     return fail(c, CAPGPU_E_INVALID, "gain_dlo / gain_step must be finite");
   if (wl->hierarchical && (wl->gain_dlo != 0.0 || wl->gain_step != 0.0))
     return fail(c, CAPGPU_E_INVALID, "gain mismatch is not supported with the hierarchical budget");
-  if (wl->controller < CAPGPU_CTRL_CAPGPU || wl->controller > CAPGPU_CTRL_CPU_ONLY)
+  if (wl->controller < CAPGPU_CTRL_CAPGPU || wl->controller > CAPGPU_CTRL_CPU_GPU)
     return fail(c, CAPGPU_E_INVALID, "controller");
   if (wl->controller != CAPGPU_CTRL_CAPGPU) {
     if (wl->hierarchical) return fail(c, CAPGPU_E_UNSUPPORTED, "baseline controllers with the hierarchical budget");
     if (wl->fs_levels < 1 || !std::isfinite(wl->safe_margin) || !(wl->p_pole >= 0.0 && wl->p_pole < 1.0))
       return fail(c, CAPGPU_E_INVALID, "baseline parameters (fs_levels >= 1, finite safe_margin, 0 <= p_pole < 1)");
+    if (wl->controller == CAPGPU_CTRL_CPU_GPU && !(wl->gpu_share > 0.0 && wl->gpu_share < 1.0))
+      return fail(c, CAPGPU_E_INVALID, "CPU+GPU needs 0 < gpu_share < 1");
   }
   if (c->prm.wmove > 0.0 && wl->hierarchical)
     return fail(c, CAPGPU_E_UNSUPPORTED, "move suppression with the hierarchical budget");

@@ -91,6 +91,7 @@ struct DevParams {
   // 1 = Fixed-step, 2 = Safe Fixed-step, 3 = GPU-only, 4 = CPU-only.
   int32_t bl_kind, bl_steps;
   double bl_margin, bl_pole;
+  double bl_share;           // CPU+GPU: GPU share of the budget (Q39)
   double wmove;              // NEXT-3 move-suppression weight W (Q36); 0 = the literal Eq. 9
   int32_t ref;               // NEXT-3 reference trajectory on (Q37): block t tracks beta + ref_w[t] (P_s - p(k))
   double ref_w[kMaxM];

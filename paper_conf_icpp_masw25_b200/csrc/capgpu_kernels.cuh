@@ -959,6 +959,11 @@ __device__ __forceinline__ double reg_get(const double (&a)[N], int j) {
 // bit-exact with the oracle).  One thread per instance, state in registers;
 // the baseline state reuses the (unused) model-state arrays: level indices in
 // mu_f, the loop command g in w, the round-robin pointer in act[0].
+// CPU+GPU's CPU meter (Q39): 0.3 C + a_0 fbar_0 + n / 2, the oracle's rounding order
+__device__ __forceinline__ double cpu_meter(double c_true, double a0, double fbar0, double noise) {
+  return __dadd_rn(__dadd_rn(__dmul_rn(0.3, c_true), __dmul_rn(a0, fbar0)), __dmul_rn(0.5, noise));
+}
+
 template <int N, int S, bool SLO>
 __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -970,7 +975,7 @@ __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, Tra
   int lev[N];
   double sumA = 0.0, g_lo = 0.0, g_hi = 0.0;
   const int kind = P.bl_kind;
-  const int j0 = kind == 3 ? 1 : 0, j1 = kind == 3 ? N : 1;
+  const int j0 = (kind == 3 || kind == 5) ? 1 : 0, j1 = (kind == 3 || kind == 5) ? N : 1;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     fbar[j] = st.fbar[j * li + i];
@@ -997,6 +1002,16 @@ __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, Tra
   const uint64_t kjit = gen_stream_key(P.seed, GEN_TAG_JIT, srv);
   const uint64_t kburst = gen_stream_key(P.seed, GEN_TAG_BURST, srv);
   const uint64_t knoise = gen_stream_key(P.seed, GEN_TAG_NOISE, srv);
+  // CPU+GPU (Q39): the CPU loop's gain and command (kept in the unused mu_p
+  // state), and the CPU meter 0.3 C + a_0 fbar_0 + n/2 of the current period,
+  // recomputed from the state and the counter-based noise of period k0
+  double Kc = 0.0, fc = 0.0, pc = 0.0;
+  if (kind == 5) {
+    Kc = __ddiv_rn(1.0 - P.bl_pole, st.A0[si]);
+    fc = st.mu_p[i];
+    if (!(fc > 0.0)) fc = P.k[0].f_min;
+    pc = cpu_meter(c_true, a_true[0], fbar[0], gen_noise(knoise, k0, P.noise_scale));
+  }
   int64_t epoch = (k0 + 1) / GEN_BURST_HOLD;
   int left = (int)(GEN_BURST_HOLD - (k0 + 1) % GEN_BURST_HOLD);
   uint32_t bmask = burst_mask<N>(P, kburst, epoch);
@@ -1041,6 +1056,15 @@ __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, Tra
       }
 #pragma unroll
       for (int j = 0; j < N; ++j) u0[j] = P.grid[P.k[j].cls * kMaxL + lev[j]].level;
+    } else if (kind == 5) {  // CPU+GPU: fixed budget split, one loop per meter
+      const double Bg = __dmul_rn(P.bl_share, cap);
+      const double Bc = __dadd_rn(cap, -Bg);
+      const double pg = __dadd_rn(p, -pc);
+      fc = fmin(fmax(__dadd_rn(fc, __dmul_rn(Kc, __dadd_rn(Bc, -pc))), P.k[0].f_min), P.k[0].f_max);
+      g = fmin(fmax(__dadd_rn(g, __dmul_rn(Kp, __dadd_rn(Bg, -pg))), g_lo), g_hi);
+      u0[0] = fc;
+#pragma unroll
+      for (int j = 1; j < N; ++j) u0[j] = fmin(fmax(g, P.k[j].f_min), P.k[j].f_max);
     } else {
       g = fmin(fmax(__dadd_rn(g, __dmul_rn(Kp, cap - p)), g_lo), g_hi);
 #pragma unroll
@@ -1090,7 +1114,9 @@ __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, Tra
     double pw = c_true;
 #pragma unroll
     for (int j = 0; j < N; ++j) pw = fma(a_true[j], fbar[j], pw);
-    p = pw + gen_noise(knoise, k + 1, P.noise_scale);
+    const double noise = gen_noise(knoise, k + 1, P.noise_scale);
+    p = pw + noise;
+    if (kind == 5) pc = cpu_meter(c_true, a_true[0], fbar[0], noise);
     if (kk >= kw) {
       sum_theta += tsum * P.inv_N;
       sum_p += p;
@@ -1110,6 +1136,7 @@ __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, Tra
   st.p[i] = p;
   st.w[i] = g;
   st.act[i] = (uint32_t)rr;
+  if (kind == 5) st.mu_p[i] = fc;
   if (tr.sum_p) tr.sum_p[i] = sum_p;
   if (tr.sumsq_p) tr.sumsq_p[i] = sumsq_p;
   if (tr.max_p) tr.max_p[i] = max_p;

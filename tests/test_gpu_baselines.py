@@ -67,3 +67,21 @@ def test_baseline_controller_is_fixed_per_simulation(G):
         g.simulate(10, G.workload_from(d2))
     g.sim_reset()
     g.simulate(10, G.workload_from(d2))
+
+
+@pytest.mark.parametrize("share,n_gpus", [(0.5, 4), (0.6, 4), (0.82, 4), (0.8, 1), (0.85, 8)])
+def test_cpu_gpu_parity(G, oracle_mod, share, n_gpus):
+    """CPU+GPU (Q39): two loops on separately metered CPU and GPU power,
+    the paper's 50/50 and 60/40 splits (P:282) and splits where both loops act;
+    chunked calls carry both loop commands and recompute the CPU meter."""
+    d = configs.baseline("cpugpu", n_servers=150, periods=240, gpu_share=share)
+    d["n_gpus"] = n_gpus
+    d["knobs"] = configs.knobs(n_gpus)
+    _compare(G, oracle_mod, d, 150, np.array([0, 70, 149]), 240, chunks=[80, 80, 80])
+
+
+def test_cpu_gpu_share_validated(G):
+    d = configs.baseline("cpugpu", n_servers=8, periods=10, gpu_share=1.0)
+    g = G.CapGPU.from_config(d, n_servers=8)
+    with pytest.raises(G.CapGPUError, match="gpu_share"):
+        g.simulate(10, G.workload_from(d))
