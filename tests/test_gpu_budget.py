@@ -1,6 +1,6 @@
 """cfg 4 hierarchical rack/cluster budget (S5, Q16) on the GPU: parity with
 the oracle's lock-step cluster simulation, and shard invariance (1 context vs
-2 and 4 loopback shards on one GPU: bitwise identical)."""
+2, 4 and 8 loopback shards on one GPU -- the 8-GPU shard logic: bitwise identical)."""
 import numpy as np
 import pytest
 import torch
@@ -45,7 +45,7 @@ def test_hierarchical_vs_oracle(G, oracle_mod, ref_alpha):
     np.testing.assert_allclose(out["final_p"], ref["final_p"], rtol=0, atol=1e-6)
 
 
-@pytest.mark.parametrize("shards", [2, 4])
+@pytest.mark.parametrize("shards", [2, 4, 8])
 def test_shard_invariance_bitwise(G, shards):
     """1 GPU holding all servers == `shards` loopback shards (same device):
     cluster aggregates, sampled traces and final powers bitwise identical."""
