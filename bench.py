@@ -150,8 +150,17 @@ def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int, single: dic
     desc = configs.by_name(cfg)
     n_inst = desc["n_servers"] * desc["workload"]["n_caps"]
     cal_p = min(periods, 100)
-    t_cal = _oracle_worker((desc, [0], cal_p))
-    if single is not None:  # the single-core rate beside the all-cores one
+    # calibration run pinned to one host core (the single-core
+    # rate is reported beside the all-cores one)
+    aff = os.sched_getaffinity(0) if hasattr(os, "sched_getaffinity") else None
+    try:
+        if aff:
+            os.sched_setaffinity(0, {min(aff)})
+        t_cal = _oracle_worker((desc, [0], cal_p))
+    finally:
+        if aff:
+            os.sched_setaffinity(0, aff)
+    if single is not None:
         single["single_core"] = cal_p / t_cal
     per_inst = t_cal / cal_p * periods
     k = max(1, int(budget_s / max(per_inst, 1e-6)))
