@@ -358,14 +358,18 @@ def main():
         peak = fp64_peak_derived()
     measured_peak = G.fp64_peak_tflops()
     traffic = None
+    ncu_pipe = None  # FP64-pipe / issue utilisation of the same kernel from the committed ncu summary
     prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}_summary.json")
     if os.path.exists(prof):
         try:
             pj = json.load(open(prof))
             if pj.get("periods") == periods and pj.get("n_inst") == n_inst:
                 traffic = pj.get("dram_bytes_per_launch")
+                ncu_pipe = {k: pj[k] for k in ("fp64_pipe_pct", "issue_active_pct", "warps_active_per_sm")
+                            if k in pj}
+                ncu_pipe = dict(ncu_pipe, source=f"profiles/ncu_cfg{args.config}_summary.json") if ncu_pipe else None
         except Exception:
-            traffic = None
+            traffic = ncu_pipe = None
 
     if rank == 0:
         if hier:
@@ -387,6 +391,8 @@ def main():
                     "fused multi-period baseline kernel k_baseline (1 launch per step)")
             par = f"dp{world} (server shards, no data-path collective)"
             launches = args.steps
+        if ncu_pipe:
+            roof["ncu"] = ncu_pipe
         line = {"metric": "server-control-steps/sec", "value": value, "unit": "server-control-steps/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": 1e3 * t_max / args.steps, "higher_is_better": True,
