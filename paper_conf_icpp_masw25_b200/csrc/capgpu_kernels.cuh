@@ -1705,6 +1705,22 @@ inline int sim_chunks(int64_t n_groups, int64_t slots, int K) {
   return best;
 }
 
+// Whether `smem` bytes of dynamic shared memory fit beside the kernel's static
+// shared memory under the device's opt-in limit.  Probed before
+// cudaFuncSetAttribute so an ineligible configuration never raises a CUDA API
+// error (compute-sanitizer reports handled API errors too).
+template <class Kern>
+bool smem_fits(Kern kern, int smem) {
+  cudaFuncAttributes fa{};
+  int dev = 0, optin = 0;
+  if (cudaFuncGetAttributes(&fa, kern) != cudaSuccess || cudaGetDevice(&dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return (size_t)smem + fa.sharedSizeBytes <= (size_t)optin;
+}
+
 template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false>
 int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int64_t k0, int K, cudaStream_t s) {
   const int smem = (int)(sizeof(double) * SlabLayout<N>::F * BLOCK);
@@ -1722,7 +1738,8 @@ int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int
       int occ = 0, dev = 0, sms = 0;
       cudaGetDevice(&dev);
       cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-      if (cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
+      if (!smem_fits(kc, smem) ||
+          cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
           cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kc, BLOCK, smem) != cudaSuccess) {
         cudaGetLastError();
         occ = 0;
@@ -1763,10 +1780,12 @@ int sim_occupancy(int block, int n_class) {
   // eligible (occupancy 0); clear the probe's error so it cannot leak
   cudaError_t e;
   if (block == 32) {
+    if (!smem_fits(k_simulate<N, M, S, 32>, smem_per_block)) return 0;
     e = cudaFuncSetAttribute(k_simulate<N, M, S, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
     if (e == cudaSuccess)
       e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 32>, 32, smem_per_block);
   } else {
+    if (!smem_fits(k_simulate<N, M, S, 128>, smem_per_block)) return 0;
     e = cudaFuncSetAttribute(k_simulate<N, M, S, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_per_block);
     if (e == cudaSuccess)
       e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_simulate<N, M, S, 128>, 128, smem_per_block);
