@@ -56,6 +56,8 @@ VARIANTS = {
     "timing": (["-DCAPGPU_PHASE_TIMING"], "_build_timing", "libcapgpu_timing.so"),
     # A/B experiments: the working tree built beside the product library
     "exp": ([], "_build_exp", "libcapgpu_exp.so"),
+    # k_period compiled for 12 resident warps per SM (read-only constants from global memory)
+    "pw12": (["-DCAPGPU_PERIOD_WARPS=12"], "_build_pw12", "libcapgpu_pw12.so"),
 }
 
 

@@ -1208,6 +1208,10 @@ __device__ __forceinline__ void cta_sum2(double a, double b, double *out_a, doub
 #define CAPGPU_PERIOD_CTA 32
 #endif
 constexpr int kPeriodCta = CAPGPU_PERIOD_CTA;
+#ifndef CAPGPU_PERIOD_WARPS
+#define CAPGPU_PERIOD_WARPS 8
+#endif
+constexpr int kPeriodWarps = CAPGPU_PERIOD_WARPS;  // resident warps per SM k_period is compiled for
 
 // Per-warp SoA tile in shared memory (field-major, 32 lanes): k_period stages
 // the server's model state and read-only constants into it with cp.async at
@@ -1226,7 +1230,9 @@ struct PeriodTile {
   // Sigma | mu_f | Sfp | A0 | thr_max | base | amp | a_true | C_true; the
   // read-only constants are staged only when the tile fits the 227 KB of
   // shared memory, else they are read from global memory where used.
-  static constexpr bool ro = (T + 7 * N + 1) * kPeriodCta * 8 <= 227 * 1024;
+  // (kPeriodWarps > 8, an experiment build: the tiles of all resident warps must fit)
+  static constexpr bool ro =
+      (T + 7 * N + 1) * kPeriodCta * 8 * (kPeriodWarps > 8 ? kPeriodWarps * 32 / kPeriodCta : 1) <= 227 * 1024;
   static constexpr int oS = 0, oMU = T, oSFP = T + N, oA0 = T + 2 * N, oTM = T + 3 * N, oBA = T + 4 * N,
                        oAM = T + 5 * N, oAT = T + 6 * N, oCT = T + 7 * N, F = ro ? T + 7 * N + 1 : T + 2 * N;
   static constexpr int bytes_per_cta = F * kPeriodCta * 8;
@@ -1438,7 +1444,7 @@ __device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs 
 // One instant of the hierarchical configuration for every local server:
 // budget caps, S1-S3, the w_i / p partial sums, S4.  State in HBM.
 template <int N, int M, int SS>
-__global__ void __launch_bounds__(kPeriodCta, 256 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
+__global__ void __launch_bounds__(kPeriodCta, kPeriodWarps * 32 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
                                                 int kk, int K) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = i < P.n_srv;
