@@ -201,7 +201,7 @@ int ora_simulate_hier(const ora_cfg *c, const ora_workload *w, int n_servers, in
                       double rack_frac, const double *W_replay, double W0_replay, int n_total, int n_tr,
                       const int64_t *tr_srv,
                       double *tr_p, double *tr_cap, double *tr_u, uint32_t *tr_active, uint32_t *tr_tie,
-                      uint8_t *tr_levels, double *agg_W, double *agg_P, double *final_p);
+                      uint8_t *tr_levels, double *tr_theta /*[N]: theta at instant k*/, double *agg_W, double *agg_P, double *final_p);
 void ora_budget_caps(int n_servers, int rack, const double *pmin, const double *w, double W,
                      double B_c, double pmin_tot, const double *B_rack_max, double *cap);
 

@@ -21,6 +21,8 @@ if _ROOT not in sys.path:
 from gen import configs  # noqa: E402
 
 LIB_PATH = os.path.join(_HERE, "libcapgpu_oracle.so")
+# tools/oracle_mutations.py points the tests at a deliberately mutated copy
+_LIB_OVERRIDE = os.environ.get("CAPGPU_ORACLE_LIB")
 SRC = [os.path.join(_HERE, "capgpu_oracle.c"), os.path.join(_HERE, "capgpu_oracle.h"),
        os.path.join(_ROOT, "gen", "capgpu_gen.h")]
 CFLAGS = ["-O2", "-fno-fast-math", "-ffp-contract=off", "-std=c11", "-Wall", "-shared", "-fPIC"]
@@ -79,8 +81,11 @@ _lib = None
 def lib():
     global _lib
     if _lib is None:
-        build()
-        L = C.CDLL(LIB_PATH)
+        if _LIB_OVERRIDE:
+            L = C.CDLL(_LIB_OVERRIDE)
+        else:
+            build()
+            L = C.CDLL(LIB_PATH)
         dp, ip = C.POINTER(C.c_double), C.POINTER(C.c_int32)
         cp = C.POINTER(OraCfg)
         L.ora_levels.argtypes = [cp, C.c_int, dp, dp, dp]
@@ -138,7 +143,7 @@ def lib():
                                             C.POINTER(C.c_uint8), dp, dp, C.POINTER(OraSummary)]
         L.ora_simulate_hier.argtypes = [cp, wp, C.c_int, C.c_int, C.c_double, C.c_double, dp, C.c_double,
                                         C.c_int, C.c_int, C.POINTER(C.c_int64), dp, dp, dp, u32p, u32p,
-                                        C.POINTER(C.c_uint8), dp, dp, dp]
+                                        C.POINTER(C.c_uint8), dp, dp, dp, dp]
         _lib = L
     return _lib
 
@@ -457,8 +462,8 @@ class Oracle:
         nt = len(tr_srv)
         out = dict(p=np.zeros((K, nt)), cap=np.zeros((K, nt)), u=np.zeros((K, nt, M, n)),
                    active=np.zeros((K, nt, M), dtype=np.uint32), tie=np.zeros((K, nt, M), dtype=np.uint32),
-                   levels=np.zeros((K, nt, S, n), dtype=np.uint8), agg_W=np.zeros(K), agg_P=np.zeros(K),
-                   final_p=np.zeros(n_servers))
+                   levels=np.zeros((K, nt, S, n), dtype=np.uint8), theta=np.zeros((K, nt, n)),
+                   agg_W=np.zeros(K), agg_P=np.zeros(K), final_p=np.zeros(n_servers))
         wr = None if W_replay is None else np.ascontiguousarray(np.asarray(W_replay, dtype=np.float64))
         u32 = C.POINTER(C.c_uint32)
         rc = self.L.ora_simulate_hier(C.byref(self.cfg), C.byref(w), n_servers, wl.get("rack", 16),
@@ -468,7 +473,8 @@ class Oracle:
                                       tr_srv.ctypes.data_as(C.POINTER(C.c_int64)), _dp(out["p"]), _dp(out["cap"]),
                                       _dp(out["u"]), out["active"].ctypes.data_as(u32),
                                       out["tie"].ctypes.data_as(u32),
-                                      out["levels"].ctypes.data_as(C.POINTER(C.c_uint8)), _dp(out["agg_W"]),
+                                      out["levels"].ctypes.data_as(C.POINTER(C.c_uint8)), _dp(out["theta"]),
+                                      _dp(out["agg_W"]),
                                       _dp(out["agg_P"]), _dp(out["final_p"]))
         if rc != 0:
             raise RuntimeError(f"ora_simulate_hier rc={rc}")
