@@ -4,7 +4,7 @@
 
 Every translation unit is compiled with
 ``-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo`` (parallel, one
-process per unit) and linked with a static CUDA runtime plus the NCCL that
+process per unit) and linked with the shared CUDA runtime plus the NCCL that
 ships with torch (site-packages/nvidia/nccl).  The host side is compiled with
 ``-ffp-contract=off`` so host-computed tables reproduce the oracle's formulas.
 """
@@ -37,6 +37,17 @@ def nccl_dirs():
         if os.path.exists(os.path.join(c, "include", "nccl.h")):
             return os.path.join(c, "include"), os.path.join(c, "lib")
     raise RuntimeError("nccl.h not found (torch's nvidia-nccl wheel)")
+
+
+def _cudart_dir():
+    """torch's libcudart.so.12 (nvidia-cuda-runtime wheel)."""
+    import importlib.util
+    spec = importlib.util.find_spec("nvidia")
+    for p in (spec.submodule_search_locations if spec else []) or []:
+        d = os.path.join(p, "cuda_runtime", "lib")
+        if os.path.exists(os.path.join(d, "libcudart.so.12")):
+            return d
+    return "/usr/local/cuda/lib64"
 
 
 def cflags():
@@ -91,8 +102,11 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None, v
     newest = max(os.path.getmtime(o) for o in objs)
     if force or not os.path.exists(lib) or os.path.getmtime(lib) < newest:
         _, libdir = nccl_dirs()
-        cmd = [NVCC, *ARCH, "-shared", "-o", lib, *objs, "-cudart", "static", f"-L{libdir}", "-l:libnccl.so.2",
-               "-Xlinker", f"-rpath,{libdir}"]
+        # shared CUDA runtime (the one torch already maps into the process, else
+        # the toolkit's): the product library carries no copy of the runtime
+        cmd = [NVCC, *ARCH, "-shared", "-o", lib, *objs, "-cudart", "shared", f"-L{libdir}", "-l:libnccl.so.2",
+               "-Xlinker", f"-rpath,{libdir}", "-Xlinker", f"-rpath,{_cudart_dir()}", "-Xlinker",
+               "-rpath,/usr/local/cuda/lib64"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr[-8000:]}")

@@ -227,6 +227,15 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   d.noise_scale = prm.noise_std * std::sqrt(3.0);
   d.inv_S = 1.0 / (double)prm.substeps;
   d.inv_lam = 1.0 / prm.lambda;
+  {
+    // fold interval of the fused kernel's scaled model state: lam^-R <= 2^600
+    // keeps Sigma' = Sigma lam^-kk and rho lam^-kk finite and lam^kk above the
+    // FTZ range of the reciprocal (a fixed 1024 overflows for lam <~ 0.5)
+    int R = 1024;
+    const double l2 = -std::log2(prm.lambda);
+    while (R > 1 && (double)R * l2 > 600.0) R >>= 1;
+    d.fold_mask = R - 1;
+  }
   d.wmove = prm.wmove;
   // Q37: block t's tracking offset is beta + ref_w[t] (P_s - p(k)), ref_w[t] =
   // mean of alpha^i over the prediction steps i whose prediction uses u_t
@@ -306,7 +315,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
 
   // ---- state workspace (SoA)
   const int64_t ni = c->n_inst, ns = c->n_srv;
-  const int64_t nd_inst = (int64_t)(5 * N + c->T + 4);
+  const int64_t nd_inst = (int64_t)(5 * N + c->T + 5);
   const int64_t nd_srv = (int64_t)(5 * N + 3);
   const int64_t grid_bytes = (int64_t)sizeof(GridEntry) * n_class * CAPGPU_MAX_LEVELS;
   const int64_t sched_words = ni + 2;  // chunked schedule of the fused kernel: counter + done[instance]
@@ -319,7 +328,16 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     return fail(nullptr, CAPGPU_E_NOMEM, "cudaMalloc(%lld): %s", (long long)bytes, cudaGetErrorString(e));
   }
   c->ws_bytes = bytes;
-  cudaMemset(c->ws, 0, (size_t)bytes);
+  // every CUDA call of create is checked: on failure nothing is left allocated
+  auto ck = [&](cudaError_t ce, const char *what) -> bool {
+    if (ce == cudaSuccess) return true;
+    cudaGetLastError();
+    fail(nullptr, CAPGPU_E_CUDA, "%s: %s", what, cudaGetErrorString(ce));
+    cudaFree(c->ws);
+    delete c;
+    return false;
+  };
+  if (!ck(cudaMemset(c->ws, 0, (size_t)bytes), "cudaMemset(workspace)")) return CAPGPU_E_CUDA;
   double *q = (double *)c->ws;
   auto take = [&](int64_t n) { double *r = q; q += n; return r; };
   StatePtrs &s = c->st;
@@ -333,6 +351,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   s.S = take(c->T * ni);
   s.Sfp = take(N * ni);
   s.cap_base = take(ni);
+  s.lamk = take(ni);
   s.a_true = take(N * ns);
   s.c_true = take(ns);
   s.thr_max = take(N * ns);
@@ -345,7 +364,8 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   q = (double *)(((uintptr_t)q + 31) & ~(uintptr_t)31);  // 16-byte vector loads of the grid table
   GridEntry *gdev = (GridEntry *)take(4 * (int64_t)n_class * CAPGPU_MAX_LEVELS);
   KnobConst *kdev = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 7) / 8);
-  cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice);
+  if (!ck(cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice), "cudaMemcpy(knobs)"))
+    return CAPGPU_E_CUDA;
   d.k_dev = kdev;
   c->kdev_slo = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS * 2 + 7) / 8);
   d.k_dev_slo[0] = c->kdev_slo;
@@ -358,8 +378,9 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     d.no_chunking = (nc && nc[0] && nc[0] != '0') ? 1 : 0;
   }
   for (int c2 = 0; c2 < n_class; ++c2)
-    cudaMemcpy(gdev + c2 * CAPGPU_MAX_LEVELS, grid[c2], sizeof(GridEntry) * CAPGPU_MAX_LEVELS,
-               cudaMemcpyHostToDevice);
+    if (!ck(cudaMemcpy(gdev + c2 * CAPGPU_MAX_LEVELS, grid[c2], sizeof(GridEntry) * CAPGPU_MAX_LEVELS,
+                       cudaMemcpyHostToDevice), "cudaMemcpy(grid)"))
+      return CAPGPU_E_CUDA;
   d.grid = gdev;
 
   if (sh.use_nccl) {
@@ -508,6 +529,26 @@ int capgpu_sim_reset(capgpu_ctx *c) {
 // e_min (f_max/level)^gamma meets SLO = ratio e_min, i.e. level >= f_max
 // ratio^(-1/gamma); bound = max(f_lo, level(q)), or f_max + SLO_INFEASIBLE when
 // no level meets it.  Validation happens before anything is launched.
+// validation of the SLO schedule alone (no side effects); *any = a ratio is set
+static int slo_validate(capgpu_ctx *c, const capgpu_workload &w, bool *any_out) {
+  bool any = false;
+  for (int j = 0; j < CAPGPU_MAX_KNOBS; ++j) {
+    if (!(w.slo_a[j] >= 0.0) || !(w.slo_b[j] >= 0.0) || !std::isfinite(w.slo_a[j]) || !std::isfinite(w.slo_b[j]))
+      return fail(c, CAPGPU_E_INVALID, "slo ratios must be finite and >= 0");
+    if (j >= c->N && (w.slo_a[j] != 0.0 || w.slo_b[j] != 0.0))
+      return fail(c, CAPGPU_E_INVALID, "slo ratio set for knob %d >= N", j);
+    any |= w.slo_a[j] != 0.0 || w.slo_b[j] != 0.0;
+  }
+  *any_out = any;
+  if (!any) return CAPGPU_OK;
+  if (w.hierarchical) return fail(c, CAPGPU_E_UNSUPPORTED, "SLO schedule with the hierarchical budget");
+  if (c->prm.wmove > 0.0 && w.controller == CAPGPU_CTRL_CAPGPU)
+    return fail(c, CAPGPU_E_UNSUPPORTED, "SLO schedule with move suppression");
+  if (w.slo_period < 0 || (w.slo_period > 0 && !(w.slo_lo >= 0 && w.slo_lo <= w.slo_hi)))
+    return fail(c, CAPGPU_E_INVALID, "slo schedule");
+  return CAPGPU_OK;
+}
+
 static int apply_slo(capgpu_ctx *c, const capgpu_workload &w, cudaStream_t s) {
   DevParams &d = c->dp;
   d.slo = 0;
@@ -590,8 +631,8 @@ static void apply_workload(DevParams &d, const capgpu_workload &w) {
 // Validation of workload + trace, first-call initialisation (plant, S0 sweep,
 // virtual period -1), base-cap override and trace slots.  Nothing is launched
 // before all arguments are validated.
-static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_trace *tr, TracePtrs &t,
-                       cudaStream_t s) {
+// Validation of one simulate call (no side effects: nothing launched or written)
+static int sim_validate(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_trace *tr, TracePtrs &t) {
   t = TracePtrs{};
   if (wl->demand_kind != 0 && wl->demand_kind != 1) return fail(c, CAPGPU_E_INVALID, "demand_kind");
   if (wl->cap_period < 0 || (wl->cap_period > 0 && !(wl->cap_lo >= 0 && wl->cap_lo <= wl->cap_hi)))
@@ -661,6 +702,14 @@ static int sim_prepare(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_tr
   }
   if (wl->cap_base_d) NEED_DEV(c, wl->cap_base_d);
   OPT_DEV(c, tr ? tr->n_miss_d : nullptr);
+  bool any_slo = false;
+  return slo_validate(c, *wl, &any_slo);
+}
+
+// Side effects of a validated simulate call: SLO bounds, workload constants,
+// first-call initialisation (identify + virtual period -1), cap bases, trace slots.
+static int sim_apply(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_trace *tr, const TracePtrs &t,
+                     cudaStream_t s) {
   {
     int rc = apply_slo(c, *wl, s);
     if (rc) return rc;
@@ -729,7 +778,9 @@ int capgpu_simulate(capgpu_ctx *c, int64_t periods, const capgpu_workload *wl, c
     return fail(c, CAPGPU_E_INVALID, "world > 1 hierarchical runs need NCCL (shard.use_nccl) or capgpu_simulate_group");
   TracePtrs t;
   cudaStream_t s = (cudaStream_t)stream;
-  int rc = sim_prepare(c, wl, tr, t, s);
+  int rc = sim_validate(c, wl, tr, t);
+  if (rc) return rc;
+  rc = sim_apply(c, wl, tr, t, s);
   if (rc) return rc;
   if (wl->hierarchical) {
     if (!c->budget.ready) {
@@ -766,11 +817,16 @@ int capgpu_simulate_group(capgpu_ctx **ctxs, int32_t n_ctx, int64_t periods, con
   }
   cudaStream_t s = (cudaStream_t)stream;
   TracePtrs t[64];
+  // every member is validated before any member is initialised or launched
   for (int q = 0; q < n_ctx; ++q) {
     capgpu_ctx *c = ctxs[q];
     if (c->wl.hierarchical && c->sim_ready && c->k_global != ctxs[0]->k_global)
       return fail(c, CAPGPU_E_ORDER, "group members are out of step");
-    int rc = sim_prepare(c, wl, trs ? trs[q] : nullptr, t[q], s);
+    int rc = sim_validate(c, wl, trs ? trs[q] : nullptr, t[q]);
+    if (rc) return rc;
+  }
+  for (int q = 0; q < n_ctx; ++q) {
+    int rc = sim_apply(ctxs[q], wl, trs ? trs[q] : nullptr, t[q], s);
     if (rc) return rc;
   }
   if (!ctxs[0]->budget.ready) {

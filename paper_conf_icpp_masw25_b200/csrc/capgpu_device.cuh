@@ -66,6 +66,8 @@ struct DevParams {
   double demand_frac;
   double q, theta_min, lam, rho, a_lo, a_hi, a_floor;
   double inv_lam;             // 1 / lam (scaled Welford state of the fused kernel)
+  int32_t fold_mask;         // R - 1: the fused kernel folds lam^-kk back into Sigma' at call periods
+                             // kk = R - 1 mod R, R = 2^r <= 1024 with lam^-R <= 2^600 (host, from lam)
   double noise_scale;        // sigma * sqrt(3) (host-computed)
   double inv_S;              // 1/S, exact (S power of two, Q22)
   double inv_N;              // 1/N for the mean-theta summary

@@ -27,6 +27,8 @@ struct StatePtrs {
   double *fbar, *acc, *thr, *p;            // plant state S4
   double *w, *mu_f, *mu_p, *S, *Sfp;       // model state S1
   double *s_prev;                          // [M] warm-start roots of the block QPs
+  double *lamk;                            // fused kernel between the chunks of one call: lam^-kk of the
+                                           // scaled model state (S, Sfp are stored scaled, see sim_run)
   uint32_t *act;                           // [M] warm-start active codes of the block QPs
   double *cap_base;                        // [1]
   int32_t *trace_slot;                     // [1] -1 = not traced
@@ -734,8 +736,8 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
   int left = (int)(GEN_BURST_HOLD - (k0 + 1) % GEN_BURST_HOLD);
   uint32_t bmask = burst_mask<N>(P, kburst, epoch);
 
-  // ---- summaries (Q25)
-  const int kw = Ktot - (4 * Ktot) / 5;
+  // ---- summaries (Q25); int64: Ktot may exceed 2^29
+  const int kw = (int)(Ktot - (4 * (int64_t)Ktot) / 5);
   double sum_p = 0.0, sumsq_p = 0.0, max_p = 0.0, sum_theta = 0.0;
   int n_viol = 0, n_miss = 0;
   if (carry) {
@@ -752,8 +754,12 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
 #pragma unroll
   for (int t = 0; t < M; ++t) act_cnt[t] = carry && tr.act_count ? __ldcg(tr.act_count + t * li + i) : 0;
 
-  // the slab holds Sigma' = Sigma / lam^kk (model_push SCALED); inv_lam_k = lam^-kk
-  double inv_lam_k = 1.0;
+  // the slab holds Sigma' = Sigma / lam^kk (model_push SCALED); inv_lam_k =
+  // lam^-kk since the last fold (call start or call period kk = R - 1 mod R).
+  // A later chunk of the same call continues the scaled representation (Sigma'
+  // and inv_lam_k carried as they are), so the chunked schedule reproduces the
+  // single-pass rounding exactly: the folds depend on the call period only.
+  double inv_lam_k = carry ? __ldcg(st.lamk + i) : 1.0;
 
   CAPGPU_PHASE_DECL
   // the loop bound is read from shared memory (item_sh[1], the same for the
@@ -763,7 +769,7 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
   for (int kk = kk0; kk < (CH ? *(const volatile int *)(item_sh + 1) : Ktot); ++kk) {  // the call's period
     const int64_t k = k0call + kk;
     const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
-    if ((kk & 1023) == 1023) {  // keep lam^-kk far from overflow: fold it back into Sigma'
+    if ((kk & P.fold_mask) == P.fold_mask) {  // keep lam^-kk far from overflow: fold it back into Sigma'
       slab_rescale<N>(my, SL::oSFP, rcp_fast(inv_lam_k));
       inv_lam_k = 1.0;
     }
@@ -860,17 +866,21 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
   li = P.n_inst;
   ls = P.n_srv;
   asm volatile("" : "+l"(i), "+l"(li), "+l"(ls), "+l"(si));
-  const double lam_k = rcp_fast(inv_lam_k);  // Sigma = lam^kk Sigma'
+  // Sigma = lam^kk Sigma' at the end of the call; between the chunks of one
+  // call Sigma' and lam^-kk are carried unchanged (bit-identical schedules)
+  const bool last = !CH || ck2.kk0 + ck2.K >= Ktot;
+  const double lam_k = last ? rcp_fast(inv_lam_k) : 1.0;
+  if (!last) __stcg(st.lamk + i, inv_lam_k);
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     __stcg(st.fbar + j * li + i, fbar[j]);
     __stcg(st.acc + j * li + i, acc[j]);
     __stcg(st.thr + j * li + i, thr[j]);
     __stcg(st.mu_f + j * li + i, MU.get(j));
-    __stcg(st.Sfp + j * li + i, SF.get(j) * lam_k);
+    __stcg(st.Sfp + j * li + i, last ? SF.get(j) * lam_k : SF.get(j));
   }
 #pragma unroll
-  for (int t = 0; t < SL::T; ++t) __stcg(st.S + t * li + i, Sm.get(t) * lam_k);
+  for (int t = 0; t < SL::T; ++t) __stcg(st.S + t * li + i, last ? Sm.get(t) * lam_k : Sm.get(t));
   __stcg(st.p + i, p);
   __stcg(st.w + i, w);
   __stcg(st.mu_p + i, mu_p);
@@ -885,7 +895,7 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
   if (tr.sum_theta) __stcg(tr.sum_theta + i, sum_theta);
   if (tr.n_viol) __stcg(tr.n_viol + i, n_viol);
   if (tr.n_miss) __stcg(tr.n_miss + i, n_miss);
-  if (tr.n_window) tr.n_window[i] = Ktot - (Ktot - (4 * Ktot) / 5);
+  if (tr.n_window) tr.n_window[i] = (int)((4 * (int64_t)Ktot) / 5);
   if (tr.final_p) tr.final_p[i] = p;
   if (tr.act_count) {
 #pragma unroll
@@ -1015,7 +1025,7 @@ __global__ void __launch_bounds__(128) k_baseline(DevParams P, StatePtrs st, Tra
   int64_t epoch = (k0 + 1) / GEN_BURST_HOLD;
   int left = (int)(GEN_BURST_HOLD - (k0 + 1) % GEN_BURST_HOLD);
   uint32_t bmask = burst_mask<N>(P, kburst, epoch);
-  const int kw = K - (4 * K) / 5;
+  const int kw = (int)(K - (4 * (int64_t)K) / 5);
   double sum_p = 0.0, sumsq_p = 0.0, max_p = 0.0, sum_theta = 0.0;
   int n_viol = 0, n_miss = 0;
   int64_t slo_r = SLO && P.slo_period > 0 ? k0 % P.slo_period : 0;
@@ -1360,7 +1370,7 @@ __device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs 
     }
     // the running summaries (read-modify-write over the window, Q25) are
     // loaded here so their latency overlaps the plant instead of following it
-    const int kw = K - (4 * K) / 5;
+    const int kw = (int)(K - (4 * (int64_t)K) / 5);
     const bool win = kk >= kw, first = kk == kw;
     double o_sum = 0.0, o_sq = 0.0, o_max = 0.0, o_th = 0.0;
     int o_viol = 0, o_ac[M];

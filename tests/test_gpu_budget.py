@@ -73,20 +73,53 @@ def test_shard_invariance_bitwise(G, shards):
         assert np.array_equal(outs[r]["tr_cap"][:, j], o1["tr_cap"][:, q])
 
 
+def _rack_budgets(d, o, n_total, theta_tr, agg_W, rack=16):
+    """B_r of the traced racks recomputed from the Q16 rule: the rack's weights
+    of instant max(k-1, 0) (w_i = mean_j theta_ij, traced on the GPU), the
+    cluster sum W of that instant (GPU all-reduce + tree) and the generator's
+    true models over the whole cluster."""
+    wl = d["workload"]
+    fmin = np.array([k["f_min"] for k in d["knobs"]])
+    fmax = np.array([k["f_max"] for k in d["knobs"]])
+    pmin, pmax = np.zeros(n_total), np.zeros(n_total)
+    for i in range(n_total):
+        g = o.gen_server(i)
+        pmin[i] = g["c_true"] + g["a_true"] @ fmin
+        pmax[i] = g["c_true"] + g["a_true"] @ fmax
+    Bc = pmin.sum() + wl["cluster_frac"] * (pmax.sum() - pmin.sum())
+    nt = theta_tr.shape[1]
+    Pr = pmin[:nt].reshape(-1, rack).sum(axis=1)
+    Brack = wl["rack_frac"] * pmax[:nt].reshape(-1, rack).sum(axis=1)
+    w = theta_tr.mean(axis=2)  # [K][nt]
+    K = w.shape[0]
+    Br = np.zeros((K, nt // rack))
+    for k in range(K):
+        kp = max(k - 1, 0)  # instant 0 uses the initial weights, whose cluster sum equals agg_W[0]
+        Wr = w[kp].reshape(-1, rack).sum(axis=1)
+        Br[k] = np.minimum(Brack, Pr + (Bc - pmin.sum()) * Wr / agg_W[kp])
+    return Br
+
+
 def test_hierarchical_replay_at_scale(G, oracle_mod):
-    """Sampled racks of a larger cluster (SURVEY §8(c.1) replay mode): the
-    oracle takes the GPU's cluster sums W(k) (checked against a full oracle run
-    above) and recomputes the first 4 racks' caps and closed loops."""
-    n, K2 = 32768, 30
+    """Sampled racks of a larger cluster (16 racks x
+    1,000 periods in replay mode): one GPU shard of cfg 4 (131,072 servers);
+    the oracle takes the GPU's cluster sums W(k) (checked against a full oracle
+    run above) and recomputes the first 16 racks' caps and closed loops.  Each
+    traced rack's caps sum to its budget B_r recomputed from the Q16 rule."""
+    n, K2 = 131072, 1000
     d = _desc(K2)
     g = G.CapGPU.from_config(d, n_servers=n, n_servers_global=n)
-    trs = np.arange(64)  # racks 0..3
+    trs = np.arange(256)  # racks 0..15
     out = {k: H(v) for k, v in g.simulate(K2, G.workload_from(d), trace_inst=trs).items()}
     W = out["agg_W"]
-    ref = oracle_mod.Oracle(d).simulate_hier(64, trs, periods=K2, W_replay=W, W0_replay=W[0], n_total=n)
+    o = oracle_mod.Oracle(d)
+    ref = o.simulate_hier(256, trs, periods=K2, W_replay=W, W0_replay=W[0], n_total=n)
     np.testing.assert_allclose(out["tr_cap"], ref["cap"], rtol=1e-10)
     np.testing.assert_allclose(out["tr_p"], ref["p"], rtol=0, atol=1e-6)
     np.testing.assert_allclose(out["tr_u"], np.transpose(ref["u"], (0, 2, 3, 1)), rtol=1e-9, atol=1e-9)
-    # per-rack conservation (Q16): the rack's caps sum to its budget B_r
-    caps = out["tr_cap"].reshape(K2, 4, 16).sum(axis=2)
-    assert np.all(caps > 0) and np.all(np.isfinite(caps))
+    assert np.array_equal(out["tr_levels"], np.transpose(ref["levels"], (0, 2, 3, 1)))
+    np.testing.assert_allclose(out["tr_theta"], np.transpose(ref["theta"], (0, 2, 1)), rtol=1e-12)
+    # per-rack conservation (Q16): each rack's caps sum to its budget B_r
+    Br = _rack_budgets(d, o, n, np.transpose(out["tr_theta"], (0, 2, 1)), W)
+    caps = out["tr_cap"].reshape(K2, 16, 16).sum(axis=2)
+    np.testing.assert_allclose(caps, Br, rtol=1e-10)
