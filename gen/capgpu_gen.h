@@ -10,8 +10,15 @@
  *   - integer splitmix64 arithmetic is exact;
  *   - uniforms are built by bit assembly (exact);
  *   - the few floating-point ops use explicit round-to-nearest intrinsics on the
- *     device (__dadd_rn / __dmul_rn, never contracted into FMA) and plain
- *     operators on the host, which must be compiled with -ffp-contract=off.
+ *     device (__dadd_rn / __dmul_rn / __fma_rn, never contracted) and plain
+ *     operators / C99 fma() on the host, which must be compiled with
+ *     -ffp-contract=off (fma() is correctly rounded: identical to __fma_rn).
+ *
+ * Per-period draws (demand jitter of every knob and the meter noise of one
+ * server and period) come from ONE splitmix64 finaliser of the (stream,
+ * period) key, expanded by a 64-bit LCG: state 1 and 2 give the four noise
+ * uniforms, state 2 + q the jitter of knobs 2q and 2q + 1 (26-bit halves).
+ * (Round 1 hashed every draw separately: ~2.5x the integer work per period.)
  *
  * Recipe citations (PAPER.md line numbers, "P:NNN"):
  *   - gains / offset of the linear power model p = A F + C: P:156-167 (Eq. 3-4)
@@ -38,9 +45,12 @@
 #if defined(__CUDA_ARCH__)
 #define GEN_ADD(a, b) __dadd_rn((a), (b))
 #define GEN_MUL(a, b) __dmul_rn((a), (b))
+#define GEN_FMA(a, b, c) __fma_rn((a), (b), (c))
 #else
+#include <math.h>
 #define GEN_ADD(a, b) ((a) + (b))
 #define GEN_MUL(a, b) ((a) * (b))
+#define GEN_FMA(a, b, c) fma((a), (b), (c))
 #endif
 
 #define GEN_MAX_KNOBS 16
@@ -48,9 +58,9 @@
 /* stream tags */
 enum {
   GEN_TAG_PARAM = 1, /* per-server constants */
-  GEN_TAG_JIT = 2,   /* per-period demand jitter */
+  GEN_TAG_JIT = 2,   /* per-period draws: demand jitter AND meter noise of period k */
   GEN_TAG_BURST = 3, /* demand bursts, held for GEN_BURST_HOLD periods */
-  GEN_TAG_NOISE = 4, /* meter noise of period k */
+  GEN_TAG_NOISE = 4, /* (unused since the per-period draws share GEN_TAG_JIT) */
   GEN_TAG_SWEEP = 5, /* meter noise of identification sweep row r */
 };
 
@@ -99,13 +109,43 @@ GEN_HD double gen_u52(uint64_t h) {
   return gen_bits_to_double(0x3FF0000000000000ULL | (h >> 12)) - 1.0;
 }
 
-/* two U26 halves of one hash, exact: x * 2^-26 */
-GEN_HD double gen_u26_hi(uint64_t h) {
-  return gen_bits_to_double(0x3FF0000000000000ULL | ((h >> 38) << 26)) - 1.0;
+/* two 26-bit uniforms of one 64-bit word as doubles in [1, 2), exact:
+ * 1 + x * 2^-26 (bits 63..38 and 37..12) */
+GEN_HD double gen_v26_hi(uint64_t h) {
+  return gen_bits_to_double(0x3FF0000000000000ULL | ((h >> 38) << 26));
 }
-GEN_HD double gen_u26_lo(uint64_t h) {
-  return gen_bits_to_double(0x3FF0000000000000ULL | (((h >> 12) & 0x3FFFFFFULL) << 26)) - 1.0;
+GEN_HD double gen_v26_lo(uint64_t h) {
+  return gen_bits_to_double(0x3FF0000000000000ULL | (((h >> 12) & 0x3FFFFFFULL) << 26));
 }
+
+/* ---------------------------------------------------------------- per-period draws */
+
+/* seed of the draws of period (or sweep row) b of a stream */
+GEN_HD uint64_t gen_period_seed(uint64_t key, int64_t b) {
+  return gen_mix64(key + (uint64_t)b * 0xD6E8FEB86659FD93ULL);
+}
+/* 64-bit LCG step (Knuth's MMIX multiplier and increment) */
+GEN_HD uint64_t gen_lcg(uint64_t x) { return x * 6364136223846793005ULL + 1442695040888963407ULL; }
+
+/* Irwin-Hall-4 noise from the period seed h: states 1 and 2 of the LCG give
+ * four 26-bit uniforms V_t in [1, 2); n = scale * (sum_t V_t - 6), i.e.
+ * scale * (U0 + U1 + U2 + U3 - 2) with U_t = V_t - 1 (mean 0, variance
+ * scale^2 / 3: scale = sigma sqrt(3)).  Sums in a fixed order. */
+GEN_HD double gen_noise_h(uint64_t h, double scale) {
+  const uint64_t s1 = gen_lcg(h), s2 = gen_lcg(s1);
+  const double a = GEN_ADD(gen_v26_hi(s1), gen_v26_lo(s1));
+  const double b = GEN_ADD(gen_v26_hi(s2), gen_v26_lo(s2));
+  return GEN_MUL(scale, GEN_ADD(GEN_ADD(a, b), -6.0));
+}
+
+/* jitter word of knob pair q (knobs 2q, 2q+1) from the period seed: LCG state 3 + q */
+GEN_HD uint64_t gen_jit_word(uint64_t h, int q) {
+  uint64_t s = gen_lcg(gen_lcg(h));
+  for (int t = 0; t <= q; ++t) s = gen_lcg(s);
+  return s;
+}
+/* jitter uniform of knob j in [1, 2) from its pair's word */
+GEN_HD double gen_jit_v(uint64_t w, int j) { return (j & 1) ? gen_v26_lo(w) : gen_v26_hi(w); }
 
 /* ---------------------------------------------------------------- params */
 
@@ -142,32 +182,31 @@ GEN_HD double gen_dem_amp(uint64_t seed, uint64_t server, int j) {
 /* Bursty demand of knob j in period k:
  *   dem = thr_max * clamp(base + amp*[U_burst(k/10) < 0.2] + 0.05*(2U_jit(k) - 1), 0, 1.5)
  * key_jit / key_burst = gen_stream_key(seed, GEN_TAG_JIT / GEN_TAG_BURST, server). */
-/* burst flag of knob j in burst epoch e = floor(k / GEN_BURST_HOLD) */
+/* burst flags of burst epoch e = floor(k / GEN_BURST_HOLD): one seed per
+ * epoch, LCG state j + 1 for knob j, flag iff its high 32 bits < 2^32 / 5
+ * (probability 0.2) */
 GEN_HD int gen_burst_flag(uint64_t key_burst, int j, int64_t epoch) {
-  return gen_u52(gen_sample(key_burst, (uint64_t)j, (uint64_t)epoch)) < 0.2;
+  uint64_t s = gen_period_seed(key_burst, epoch);
+  for (int t = 0; t <= j; ++t) s = gen_lcg(s);
+  return (uint32_t)(s >> 32) < 858993460u;
 }
 
-/* jitter uniform of knob j in period k: knobs 2q and 2q+1 share one hash
- * (26-bit halves), so a server draws ceil(N/2) jitter hashes per period */
-GEN_HD uint64_t gen_jit_hash(uint64_t key_jit, int pair, int64_t k) {
-  return gen_sample(key_jit, (uint64_t)pair, (uint64_t)k);
-}
-GEN_HD double gen_jit_u(uint64_t h, int j) { return (j & 1) ? gen_u26_lo(h) : gen_u26_hi(h); }
-
-/* demand from the jitter uniform and the burst flag:
- * thr_max * clamp(base + amp*burst + 0.05 (2u - 1), 0, 1.5) */
-GEN_HD double gen_demand_u(double uj, int burst, double thr_max, double base, double amp) {
+/* demand from the jitter uniform v in [1, 2) and the burst flag:
+ *   thr_max * min(base + amp*burst + (0.1 v - 0.15), 1.5)
+ * (jitter 0.05 (2U - 1) with U = v - 1, one correctly rounded fma; the lower
+ * clamp at 0 of the recipe never binds: base >= 0.2 > 0.05) */
+GEN_HD double gen_demand_u(double v, int burst, double thr_max, double base, double amp) {
   double x = burst ? GEN_ADD(base, amp) : base;
-  double t = GEN_ADD(GEN_MUL(2.0, uj), -1.0);
-  double y = GEN_ADD(x, GEN_MUL(0.05, t));
-  y = y < 0.0 ? 0.0 : (y > 1.5 ? 1.5 : y);
+  double y = GEN_ADD(x, GEN_FMA(0.1, v, -0.15));
+  y = y > 1.5 ? 1.5 : y;
   return GEN_MUL(thr_max, y);
 }
 
 /* demand given the burst flag of the period's epoch */
 GEN_HD double gen_demand_flag(uint64_t key_jit, int j, int64_t k, int burst, double thr_max,
                               double base, double amp) {
-  return gen_demand_u(gen_jit_u(gen_jit_hash(key_jit, j >> 1, k), j), burst, thr_max, base, amp);
+  const uint64_t w = gen_jit_word(gen_period_seed(key_jit, k), j >> 1);
+  return gen_demand_u(gen_jit_v(w, j), burst, thr_max, base, amp);
 }
 
 GEN_HD double gen_demand_bursty(uint64_t key_jit, uint64_t key_burst, int j, int64_t k,
@@ -182,13 +221,11 @@ GEN_HD double gen_demand_const(double thr_max, double frac) { return GEN_MUL(thr
 /* ---------------------------------------------------------------- noise */
 
 /* Irwin-Hall-4 meter noise with standard deviation sigma (scale = sigma*sqrt(3),
- * computed once on the host): n = scale * (U0 + U1 + U2 + U3 - 2), U_t = 26-bit
- * uniforms from two hashes.  Sample slot b is the period k (or sweep row r). */
+ * computed once on the host) of slot b of a stream: the period k of the
+ * GEN_TAG_JIT stream (shared with the demand jitter of period k) or the row r
+ * of the identification sweep stream (GEN_TAG_SWEEP). */
 GEN_HD double gen_noise(uint64_t key, int64_t b, double scale) {
-  uint64_t h0 = gen_sample(key, 0, (uint64_t)b);
-  uint64_t h1 = gen_sample(key, 1, (uint64_t)b);
-  double s = GEN_ADD(GEN_ADD(GEN_ADD(gen_u26_hi(h0), gen_u26_lo(h0)), gen_u26_hi(h1)), gen_u26_lo(h1));
-  return GEN_MUL(scale, GEN_ADD(s, -2.0));
+  return gen_noise_h(gen_period_seed(key, b), scale);
 }
 
 /* ---------------------------------------------------------------- caps */

@@ -90,7 +90,9 @@ typedef struct {
   uint64_t seed;      /* synthetic-input seed */
   double wmove;       /* NEXT-3 move suppression (Q36): Eq. 9 + sum_{t<M} wmove |d(k+t|k)|^2,
                          >= 0 (W^2/MHz^2); 0 = the literal Eq. 9.  > 0 couples the M blocks: solved by a
-                         generic per-instance active set, CUDA path for M * N <= 10, capgpu_simulate only
+                         per-instance active set on the block-tridiagonal Hessian (Woodbury: N tridiagonal
+                         M x M solves + one M x M system per iteration), CUDA path for M * N <= 36,
+                         capgpu_simulate only
                          (not control_step / hierarchical / SLO schedule: CAPGPU_E_UNSUPPORTED) */
   double ref_alpha;   /* NEXT-3 reference trajectory ("a reference trajectory"; Q37):
                          prediction step i tracks r(k+i|k) = P_s - ref_alpha^i (P_s - p(k)) instead of

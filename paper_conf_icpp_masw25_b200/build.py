@@ -89,13 +89,28 @@ def _compile(src: str, force: bool, verbose: bool, bdir: str = BUILD, extra=()) 
     return obj
 
 
-def build(force: bool = False, verbose: bool = False, jobs: int | None = None, variant: str | None = None) -> str:
+def build(force: bool = False, verbose: bool = False, jobs: int | None = None, variant: str | None = None,
+          defs: tuple = ()) -> str:
     extra, bdir, lib = ((), BUILD, LIB)
+    if variant and variant not in VARIANTS:  # ad-hoc experiment build: --variant=NAME --defs="-DX -DY"
+        VARIANTS[variant] = (list(defs), f"_build_{variant}", f"libcapgpu_{variant}.so")
     if variant:
         flags, sub, name = VARIANTS[variant]
         extra, bdir, lib = (flags, os.path.join(PKG, sub), os.path.join(PKG, name))
     os.makedirs(bdir, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    # a library newer than every source is current even without its objects
+    # (the object directory does not travel to the GPU box)
+    if not force and os.path.exists(lib) and os.path.getmtime(lib) >= max(
+            os.path.getmtime(d) for d in _deps() + srcs + [os.path.abspath(__file__)]):
+        return lib
+    only = [int(x) for x in os.environ.get("CAPGPU_ONLY_N", "").split(",") if x] if variant else []
+    if only:  # experiment build with a subset of the knob counts (smaller library to ship)
+        srcs = [s_ for s_ in srcs if not os.path.basename(s_).startswith("inst_n") or
+                int(os.path.basename(s_)[6:-3]) in only]
+        extra = list(extra) + ["-DCAPGPU_SUBSET"] + [
+            f"-DCAPGPU_CASE_IF_{n}=" + (f"case {n}: return launchers_n{n}(M);" if n in only else "")
+            for n in range(2, 17)]
     jobs = jobs or max(1, min(len(srcs), os.cpu_count() or 4))
     with cf.ThreadPoolExecutor(jobs) as ex:
         objs = list(ex.map(lambda s: _compile(s, force, verbose, bdir, extra), srcs))
@@ -115,4 +130,5 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None, v
 
 if __name__ == "__main__":
     var = next((a.split("=", 1)[1] for a in sys.argv if a.startswith("--variant=")), None)
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, variant=var))
+    defs = next((a.split("=", 1)[1].split() for a in sys.argv if a.startswith("--defs=")), [])
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, variant=var, defs=tuple(defs)))

@@ -78,22 +78,18 @@ static bool is_device_ptr(const void *p) {
   } while (0)
 
 static Launchers launchers(int N, int M) {
+  // experiment builds may compile a subset of the knob counts (build.py --only-n)
+#ifdef CAPGPU_SUBSET
+#define CAPGPU_CASE(NN) CAPGPU_CASE_IF_##NN
+#else
+#define CAPGPU_CASE(NN) \
+  case NN: return launchers_n##NN(M);
+#endif
   switch (N) {
-    case 2: return launchers_n2(M);
-    case 3: return launchers_n3(M);
-    case 4: return launchers_n4(M);
-    case 5: return launchers_n5(M);
-    case 6: return launchers_n6(M);
-    case 7: return launchers_n7(M);
-    case 8: return launchers_n8(M);
-    case 9: return launchers_n9(M);
-    case 10: return launchers_n10(M);
-    case 11: return launchers_n11(M);
-    case 12: return launchers_n12(M);
-    case 13: return launchers_n13(M);
-    case 14: return launchers_n14(M);
-    case 15: return launchers_n15(M);
-    case 16: return launchers_n16(M);
+    CAPGPU_CASE(2) CAPGPU_CASE(3) CAPGPU_CASE(4) CAPGPU_CASE(5) CAPGPU_CASE(6) CAPGPU_CASE(7) CAPGPU_CASE(8)
+    CAPGPU_CASE(9) CAPGPU_CASE(10) CAPGPU_CASE(11) CAPGPU_CASE(12) CAPGPU_CASE(13) CAPGPU_CASE(14)
+    CAPGPU_CASE(15) CAPGPU_CASE(16)
+#undef CAPGPU_CASE
     default: return Launchers{};
   }
 }
@@ -307,7 +303,16 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
     k.span = k.hi - k.m;
     k.r0 = b.r0 == 0.0 ? prm.r0 : b.r0;
     k.inv_r0 = 1.0 / k.r0;
+    k.pos_tol = 1e-9;  // grid steps: >> the table and sub-step rounding (ulps of f_max; plant_pair)
   }
+  // two-level pair tables of plant_pair: row l = {mid(l), level(l), level(l+1), g(l), g(l+1)}
+  PairEntry pairs[CAPGPU_MAX_KNOBS][CAPGPU_MAX_LEVELS];
+  for (int c2 = 0; c2 < n_class; ++c2)
+    for (int l = 0; l < CAPGPU_MAX_LEVELS; ++l) {
+      const int l0 = l + 1 < CAPGPU_MAX_LEVELS ? l : l - 1;
+      const GridEntry &a = grid[c2][l0], &b = grid[c2][l0 + 1];
+      pairs[c2][l] = PairEntry{a.mid_hi, a.level, b.level, a.g, b.g, 0.0};
+    }
   d.convex = 1;
   for (int j = 0; j < N; ++j) d.convex &= d.k[j].lo == d.k[j].m ? 1 : 0;
   c->convex_static = d.convex;
@@ -317,7 +322,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   const int64_t ni = c->n_inst, ns = c->n_srv;
   const int64_t nd_inst = (int64_t)(5 * N + c->T + 5);
   const int64_t nd_srv = (int64_t)(5 * N + 3);
-  const int64_t grid_bytes = (int64_t)sizeof(GridEntry) * n_class * CAPGPU_MAX_LEVELS;
+  const int64_t grid_bytes = (int64_t)(sizeof(GridEntry) + sizeof(PairEntry)) * n_class * CAPGPU_MAX_LEVELS;
   const int64_t sched_words = ni + 2;  // chunked schedule of the fused kernel: counter + done[instance]
   const int64_t bytes = 8 * (nd_inst * ni + nd_srv * ns) + 12 * (int64_t)h.M * ni + 4 * ni + 4 * sched_words +
                         grid_bytes + (int64_t)sizeof(KnobConst) * CAPGPU_MAX_KNOBS * 3 + 256;
@@ -363,6 +368,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   s.s_prev = take((int64_t)h.M * ni);
   q = (double *)(((uintptr_t)q + 31) & ~(uintptr_t)31);  // 16-byte vector loads of the grid table
   GridEntry *gdev = (GridEntry *)take(4 * (int64_t)n_class * CAPGPU_MAX_LEVELS);
+  PairEntry *pdev = (PairEntry *)take(6 * (int64_t)n_class * CAPGPU_MAX_LEVELS);
   KnobConst *kdev = (KnobConst *)take((int64_t)(sizeof(KnobConst) * CAPGPU_MAX_KNOBS + 7) / 8);
   if (!ck(cudaMemcpy(kdev, d.k, sizeof(KnobConst) * CAPGPU_MAX_KNOBS, cudaMemcpyHostToDevice), "cudaMemcpy(knobs)"))
     return CAPGPU_E_CUDA;
@@ -382,6 +388,11 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
                        cudaMemcpyHostToDevice), "cudaMemcpy(grid)"))
       return CAPGPU_E_CUDA;
   d.grid = gdev;
+  for (int c2 = 0; c2 < n_class; ++c2)
+    if (!ck(cudaMemcpy(pdev + c2 * CAPGPU_MAX_LEVELS, pairs[c2], sizeof(PairEntry) * CAPGPU_MAX_LEVELS,
+                       cudaMemcpyHostToDevice), "cudaMemcpy(pairs)"))
+      return CAPGPU_E_CUDA;
+  d.pair = pdev;
 
   if (sh.use_nccl) {
     int rc = budget_init_nccl(c->budget, sh.nccl_id, sh.world, sh.rank, c->err);

@@ -45,6 +45,7 @@ struct KnobConst {
   double lo, hi, m;                     // box [l, h] (Eq. 10a, Q14) and penalty reference f_min (Q7)
   double span;                          // hi - m
   double r0, inv_r0;                    // r0_j and 1 / r0_j (Q6, Q9)
+  double pos_tol;                       // plant_pair: distance to an interior grid point (in steps) that forces the exact path
   int32_t L;                            // levels
   int32_t sweep_base;
   int32_t cls;                          // grid class (knobs with identical grids share a table)
@@ -55,6 +56,14 @@ struct KnobConst {
 // level(l), g(l)}: decision thresholds, frequency and capacity factor (Q14, Q15).
 struct GridEntry {
   double mid_lo, mid_hi, level, g;
+};
+
+// Per-class table of neighbouring level pairs (l, l+1), l = 0..L-2: the
+// threshold mid(l) between them, both levels and both capacity factors --
+// the same host-computed values as GridEntry (oracle formulas).  Row L-1
+// duplicates row L-2 (never indexed).
+struct PairEntry {
+  double mid, lev0, lev1, g0, g1, pad;
 };
 
 struct DevParams {
@@ -79,6 +88,7 @@ struct DevParams {
   int64_t srv_begin;         // global id of local server 0
   int64_t n_srv, n_inst;     // local counts
   const GridEntry *grid;     // device [n_class][kMaxL]
+  const PairEntry *pair;     // device [n_class][kMaxL] (plant_pair)
   const KnobConst *k_dev;    // device copy of k[] for out-of-line code (keeps P in the param bank)
   // SLO schedule (NEXT-1, §6.4, Eq. 10b-c; Q29-Q31).  Phase B at instant k
   // while slo_period > 0 and k mod slo_period in [slo_lo, slo_hi).  k_dev_slo[ph]
@@ -141,6 +151,15 @@ __device__ __forceinline__ double rcp_fast(double x) {
   return fma(y, fma(e, e, e), y);
 }
 
+// One Newton step on the MUFU seed: |rel. error| <= e^2 < 2^-39 (~2e-12).
+// Only for quantities whose error enters the outputs linearly and far below
+// the 1e-9 parity bar (the weights theta that scale the MPC penalties).
+__device__ __forceinline__ double rcp_nr1(double x) {
+  double y;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
+  return fma(y, fma(-x, y, 1.0), y);
+}
+
 __device__ __forceinline__ long long dbits(double x) { return __double_as_longlong(x); }
 __device__ __forceinline__ double bitsd(long long b) { return __longlong_as_double(b); }
 
@@ -159,9 +178,9 @@ __device__ __forceinline__ double pclamp(double x, double lo, double hi) {
 // the solve uses rho / Lambda (same solution), and the caller multiplies
 // Sigma' back by Lambda before it leaves the kernel (and every 1024 periods).
 // SCALED = false: the plain form above (state in HBM, one period per launch).
-template <int N, bool SCALED, class SAcc, class VAcc>
+template <int N, bool SCALED, class SAcc, class VAcc, class FAcc>
 __device__ __forceinline__ void model_push(double lam, double inv_lam_k, double &w, VAcc mu_f, double &mu_p,
-                                           SAcc S, VAcc Sfp, const double (&f)[N], double p) {
+                                           SAcc S, FAcc Sfp, const double (&f)[N], double p) {
   w = fma(lam, w, 1.0);
   const double iw = rcp_fast(w);
   const double e = SCALED ? (1.0 - iw) * inv_lam_k : 1.0 - iw;
@@ -602,6 +621,228 @@ __device__ __forceinline__ uint32_t move_qp(const DevParams &P, const KnobConst 
   return status;
 }
 
+// ------------------------------------------------------------------ S3 move suppression, structured (NEXT-3, M N <= 64)
+// The same QP as move_qp (Q36), solved without forming the MN x MN Hessian.
+// H = T + sum_t c_t v_t v_t^T: T is N independent M x M tridiagonal matrices
+// (knob j: diagonal R_j + W (1 + [t < M-1]), off-diagonal -W between t and
+// t + 1) and v_t = A on block t (the rank-1 tracking term of Eq. 9's block t).
+// The equality-constrained subproblem of each active-set iteration keeps this
+// form on the free variables (fixed rows -> identity, their couplings -> the
+// right-hand side), so it is solved by the Woodbury identity:
+//   y = T^-1 r - T^-1 V (C^-1 + V^T T^-1 V)^-1 V^T T^-1 r,
+// N tridiagonal solves of size M plus one M x M system: O(M^2 N) per
+// iteration instead of the dense O((MN)^3 / 6).  T is strictly diagonally
+// dominant (R > 0) and the M x M capacitance matrix is SPD.
+
+// LDL^T of one knob's masked tridiagonal (free: diagonal dd_t, coupling -W
+// to a free neighbour; fixed: identity row) and its inverse G (symmetric).
+template <int M>
+__device__ __forceinline__ void tri_inverse(const double (&dd)[M], const bool (&fr)[M], double W, double (&G)[M][M],
+                                            double (&dinv)[M], double (&ll)[M]) {
+  // factor: D_0 = dd_0; l_t = e_t / D_{t-1}; D_t = dd_t - e_t l_t, e_t = -W if t-1, t both free
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+    const double e = (t > 0 && fr[t] && fr[t - 1]) ? -W : 0.0;
+    const double Dt = fr[t] ? (t > 0 ? fma(-e, e * dinv[t > 0 ? t - 1 : 0], dd[t]) : dd[t]) : 1.0;
+    ll[t] = t > 0 ? e * dinv[t > 0 ? t - 1 : 0] : 0.0;
+    dinv[t] = rcp_fast(Dt);
+  }
+  // columns of the inverse: solve L D L^T g = e_c
+#pragma unroll
+  for (int c = 0; c < M; ++c) {
+    double y[M];
+#pragma unroll
+    for (int t = 0; t < M; ++t) y[t] = (t == c ? 1.0 : 0.0) - (t > 0 ? ll[t] * y[t > 0 ? t - 1 : 0] : 0.0);
+#pragma unroll
+    for (int t = M - 1; t >= 0; --t) G[t][c] = y[t] * dinv[t] - (t < M - 1 ? ll[t < M - 1 ? t + 1 : 0] * G[t < M - 1 ? t + 1 : 0][c] : 0.0);
+  }
+}
+
+template <int M>
+__device__ __forceinline__ void tri_solve(const double (&dinv)[M], const double (&ll)[M], const double (&b)[M],
+                                          double (&x)[M]) {
+  double y[M];
+#pragma unroll
+  for (int t = 0; t < M; ++t) y[t] = b[t] - (t > 0 ? ll[t] * y[t > 0 ? t - 1 : 0] : 0.0);
+#pragma unroll
+  for (int t = M - 1; t >= 0; --t) x[t] = y[t] * dinv[t] - (t < M - 1 ? ll[t < M - 1 ? t + 1 : 0] * x[t < M - 1 ? t + 1 : 0] : 0.0);
+}
+
+template <int N, int M>
+__device__ __forceinline__ uint32_t move_qp_w(const DevParams &P, const KnobConst *kc, const double (&a)[N],
+                                              const double (&R)[N], double beta, double dref, const double (&f)[N],
+                                              uint32_t (&act)[M], double (&x)[M * N]) {
+  constexpr int V = M * N;
+  static_assert(V <= 64, "masks are 64-bit");
+  const double W = P.wmove;
+  double g[V];
+  uint64_t lo_m = 0u, up_m = 0u;  // working set: variable fixed at its lower / upper bound
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const int v = t * N + j;
+      g[v] = P.ct[t] * fma(P.ref_w[t], dref, beta) * a[j] - R[j] * kc[j].m - (t == 0 ? W * f[j] : 0.0);
+      const uint32_t code = (act[t] >> (2 * j)) & 3u;
+      lo_m |= (code == 1u ? 1ull : 0ull) << v;
+      up_m |= (code == 2u ? 1ull : 0ull) << v;
+      x[v] = code == 1u ? kc[j].lo : (code == 2u ? kc[j].hi : pclamp(f[j], kc[j].lo, kc[j].hi));
+    }
+  }
+  double gscale = 1.0;
+#pragma unroll
+  for (int v = 0; v < V; ++v) gscale = fmax(gscale, fabs(g[v]));
+  double cinv[M];
+#pragma unroll
+  for (int t = 0; t < M; ++t) cinv[t] = 1.0 / P.ct[t];
+  uint32_t status = CAPGPU_ST_SOLVER_CAP;
+#pragma unroll 1
+  for (int it = 0; it < 3 * V + 3; ++it) {
+    const uint64_t fix = lo_m | up_m;
+    // rank-1 loads of the fixed variables per block: sX_t = sum_{j fixed at t} A_j x_tj
+    double sX[M];
+#pragma unroll
+    for (int t = 0; t < M; ++t) {
+      sX[t] = 0.0;
+#pragma unroll
+      for (int j = 0; j < N; ++j)
+        if ((fix >> (t * N + j)) & 1ull) sX[t] = fma(a[j], x[t * N + j], sX[t]);
+    }
+    // pass 1, per knob: p_j = T_j^-1 r_j, Q += (a_j a_j^T) o G_j on the free entries, q = V^T p
+    double Q[M][M], q[M];
+#pragma unroll
+    for (int s2 = 0; s2 < M; ++s2) {
+      q[s2] = 0.0;
+#pragma unroll
+      for (int t = 0; t < M; ++t) Q[s2][t] = 0.0;
+    }
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      double dd[M], r[M], G[M][M], dinv[M], ll[M], pj[M];
+      bool fr[M];
+#pragma unroll
+      for (int t = 0; t < M; ++t) {
+        const int v = t * N + j;
+        fr[t] = !((fix >> v) & 1ull);
+        dd[t] = R[j] + W * (t < M - 1 ? 2.0 : 1.0) + 0.0;
+        // r = -g - H[:, fixed] x_fixed on the free rows: tridiagonal couplings
+        // (-W to a fixed neighbour) and the block's rank-1 term
+        double rv = -g[v] - P.ct[t] * a[j] * sX[t];
+        if (t > 0 && ((fix >> (v >= N ? v - N : 0)) & 1ull)) rv = fma(W, x[v >= N ? v - N : 0], rv);
+        if (t < M - 1 && ((fix >> (v + N < V ? v + N : 0)) & 1ull)) rv = fma(W, x[v + N < V ? v + N : 0], rv);
+        r[t] = fr[t] ? rv : 0.0;
+      }
+      tri_inverse<M>(dd, fr, W, G, dinv, ll);
+      tri_solve<M>(dinv, ll, r, pj);
+#pragma unroll
+      for (int s2 = 0; s2 < M; ++s2) {
+        const double as = fr[s2] ? a[j] : 0.0;
+        q[s2] = fma(as, pj[s2], q[s2]);
+#pragma unroll
+        for (int t = 0; t < M; ++t) Q[s2][t] = fma(as * (fr[t] ? a[j] : 0.0), G[s2][t], Q[s2][t]);
+      }
+    }
+    // capacitance system (C^-1 + Q) z = q, M x M SPD: plain LDL^T
+    double z[M];
+    {
+      double L[Tri<M>::size], b[M];
+#pragma unroll
+      for (int s2 = 0; s2 < M; ++s2) {
+        b[s2] = q[s2];
+#pragma unroll
+        for (int t = s2; t < M; ++t) L[Tri<M>::idx(s2, t)] = Q[s2][t] + (s2 == t ? cinv[s2] : 0.0);
+      }
+      ldlt_solve<M>(L, b, z);
+    }
+    // pass 2, per knob: y_j = p_j - T_j^-1 (a_j z) on the free entries
+    double xs[V];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      double dd[M], r[M], G[M][M], dinv[M], ll[M], pj[M], c[M], cj[M];
+      bool fr[M];
+#pragma unroll
+      for (int t = 0; t < M; ++t) {
+        const int v = t * N + j;
+        fr[t] = !((fix >> v) & 1ull);
+        dd[t] = R[j] + W * (t < M - 1 ? 2.0 : 1.0) + 0.0;
+        double rv = -g[v] - P.ct[t] * a[j] * sX[t];
+        if (t > 0 && ((fix >> (v >= N ? v - N : 0)) & 1ull)) rv = fma(W, x[v >= N ? v - N : 0], rv);
+        if (t < M - 1 && ((fix >> (v + N < V ? v + N : 0)) & 1ull)) rv = fma(W, x[v + N < V ? v + N : 0], rv);
+        r[t] = fr[t] ? rv : 0.0;
+        c[t] = fr[t] ? a[j] * z[t] : 0.0;
+      }
+      tri_inverse<M>(dd, fr, W, G, dinv, ll);
+      tri_solve<M>(dinv, ll, r, pj);
+      tri_solve<M>(dinv, ll, c, cj);
+#pragma unroll
+      for (int t = 0; t < M; ++t) xs[t * N + j] = fr[t] ? pj[t] - cj[t] : x[t * N + j];
+    }
+    // ratio test along xs - x over the free variables
+    double alpha = 1.0;
+    int blk = -1;
+    bool blk_up = false;
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      if ((fix >> u) & 1ull) continue;
+      const int j = u % N;
+      const double d = xs[u] - x[u];
+      if (xs[u] < kc[j].lo && d < 0.0) {
+        const double al = (kc[j].lo - x[u]) / d;
+        if (al < alpha) { alpha = al; blk = u; blk_up = false; }
+      } else if (xs[u] > kc[j].hi && d > 0.0) {
+        const double al = (kc[j].hi - x[u]) / d;
+        if (al < alpha) { alpha = al; blk = u; blk_up = true; }
+      }
+    }
+    if (blk >= 0) {  // blocked: step to the bound, fix the blocking variable
+#pragma unroll
+      for (int u = 0; u < V; ++u)
+        if (!((fix >> u) & 1ull)) x[u] = pclamp(fma(alpha, xs[u] - x[u], x[u]), kc[u % N].lo, kc[u % N].hi);
+      x[blk] = blk_up ? kc[blk % N].hi : kc[blk % N].lo;
+      if (blk_up) up_m |= 1ull << blk; else lo_m |= 1ull << blk;
+      continue;
+    }
+#pragma unroll
+    for (int u = 0; u < V; ++u) x[u] = xs[u];
+    // stationary on the face: bound multipliers of the fixed variables,
+    // grad = g + H x = g + T x + c_t A_j (A . x_t)
+    double ax[M];
+#pragma unroll
+    for (int t = 0; t < M; ++t) {
+      ax[t] = 0.0;
+#pragma unroll
+      for (int j = 0; j < N; ++j) ax[t] = fma(a[j], x[t * N + j], ax[t]);
+    }
+    int worst = -1;
+    double most = -1e-12 * gscale;
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      if (!((fix >> u) & 1ull)) continue;
+      const int t = u / N, j = u % N;
+      double gr = fma(P.ct[t] * a[j], ax[t], g[u]);
+      gr = fma(R[j] + W * (t < M - 1 ? 2.0 : 1.0), x[u], gr);
+      if (t > 0) gr = fma(-W, x[u >= N ? u - N : 0], gr);
+      if (t < M - 1) gr = fma(-W, x[u + N < V ? u + N : 0], gr);
+      const double lam = ((lo_m >> u) & 1ull) ? gr : -gr;
+      if (lam < most) { most = lam; worst = u; }
+    }
+    if (worst < 0) { status = 0u; break; }
+    lo_m &= ~(1ull << worst);
+    up_m &= ~(1ull << worst);
+  }
+#pragma unroll
+  for (int t = 0; t < M; ++t) {
+    uint32_t c = 0u;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const int v = t * N + j;
+      c |= ((((lo_m >> v) & 1ull) ? 1u : 0u) | (((up_m >> v) & 1ull) ? 2u : 0u)) << (2 * j);
+    }
+    act[t] = c;
+  }
+  return status;
+}
+
 // ------------------------------------------------------------------ S4 plant
 // First-order delta-sigma over S sub-steps, period averages (Q22),
 // throughput min(dem, thr_max g(l)) (Q18).  Exact arithmetic (no contraction;
@@ -704,6 +945,127 @@ __device__ __forceinline__ void plant_delta_sigma_c(const DevParams &P, const Gr
     thr[j] = __dmul_rn(ts, P.inv_S);
   }
   if constexpr (MISS) *miss += nm;
+}
+
+// plant_pair: the same delta-sigma plant, bit for bit, with two candidate
+// levels per knob and period instead of three.
+//
+// Why two suffice.  |acc| <= step/2 (+ a few ulps of the host's table
+// rounding) after every sub-step, so every sub-step value v = u + acc lies
+// within step/2 (+ ulps) of the period's command u.  Let l = floor of u's
+// grid position (u - f_min)/step, clamped to [0, L-2]: when u is farther
+// than pos_tol steps (1e-9, >> the ulps) from the grid points level(l) and
+// level(l+1), no v can reach the thresholds mid(l-1) or mid(l+1), so the
+// level index #{mid < v} of the oracle is l + [v > mid(l)] -- one compare,
+// one two-way select of the level and of the served throughput per sub-step.
+// At the grid ends (l = 0, l + 1 = L-1) there is no outer threshold, so a
+// command sitting ON f_min or f_max (a knob at a bound: the common case) is
+// still a two-level case.  A command within pos_tol of an interior grid
+// point (rare unless an SLO bound is an interior level, which runs
+// plant_delta_sigma_c) takes the generic three-way plant for the whole
+// instance (out of line).  Same operations in the same order as the oracle
+// (v = u + acc, acc = v - level, sums in ascending s): identical bits.
+template <int N>
+__device__ __noinline__ void plant_generic_ool(const KnobConst *k_dev, int S, double inv_S, const GridEntry *grid,
+                                               const double *u0, double *acc, const double *dem,
+                                               const double *thr_max, double *fbar, double *thr) {
+  for (int j = 0; j < N; ++j) {
+    const KnobConst &kc = k_dev[j];
+    const GridEntry *tab = grid + kc.cls * kMaxL;
+    double a = acc[j], fs = 0.0, ts = 0.0;
+    for (int s = 0; s < S; ++s) {
+      const double v = __dadd_rn(u0[j], a);
+      const int l = level_of<N>(kc, tab, v);
+      const double lev = tab[l].level;
+      a = __dadd_rn(v, -lev);
+      fs = __dadd_rn(fs, lev);
+      const double capj = __dmul_rn(thr_max[j], tab[l].g);
+      ts = __dadd_rn(ts, dem[j] < capj ? dem[j] : capj);
+    }
+    acc[j] = a;
+    fbar[j] = __dmul_rn(fs, inv_S);
+    thr[j] = __dmul_rn(ts, inv_S);
+  }
+}
+
+// Grid position of u in steps, rounded to the nearest integer without a
+// float->int conversion: r = (x + 1.5 2^52) - 1.5 2^52 is rint(x) exactly for
+// |x| < 2^51 and the low word of x + 1.5 2^52 is rint(x) as an integer.
+struct GridPos {
+  int ln;     // rint(x)
+  double d;   // x - rint(x) in [-1/2, 1/2]
+};
+__device__ __forceinline__ GridPos grid_pos(double u, const KnobConst &kc) {
+  const double x = (u - kc.f_min) * kc.inv_step;
+  const double magic = 6755399441055744.0;
+  const double xm = x + magic;
+  return GridPos{(int)__double2loint(xm), x - (xm - magic)};
+}
+
+// one knob over S sub-steps on the pair (lev0 | lev1 above mid), from acc
+template <int S>
+__device__ __forceinline__ void pair_substeps(double u, double &acc, double mid, double lev0, double lev1, double t0,
+                                              double t1, double inv_S, double &fbar, double &thr) {
+  double a = acc, fs, ts;
+#pragma unroll
+  for (int s = 0; s < S; ++s) {
+    const double v = __dadd_rn(u, a);
+    const bool up = v > mid;
+    const double lev = up ? lev1 : lev0;
+    const double tt = up ? t1 : t0;
+    a = __dadd_rn(v, -lev);
+    // s = 0: 0 + x = x exactly (x >= 0), so the oracle's first add is a copy
+    fs = s == 0 ? lev : __dadd_rn(fs, lev);
+    ts = s == 0 ? tt : __dadd_rn(ts, tt);
+  }
+  acc = a;
+  fbar = __dmul_rn(fs, inv_S);
+  thr = __dmul_rn(ts, inv_S);
+}
+
+template <int N, int S>
+__device__ __forceinline__ void plant_pair(const DevParams &P, const double (&u0)[N], double (&acc)[N],
+                                           const double (&dem)[N], const double (&thr_max)[N], double (&fbar)[N],
+                                           double (&thr)[N]) {
+  static_assert(S >= 1, "compile-time sub-steps");
+  int lidx[N];
+  bool exc = false;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    const KnobConst &kc = P.k[j];
+    const GridPos g = grid_pos(u0[j], kc);
+    exc |= fabs(g.d) < kc.pos_tol && g.ln > 0 && g.ln < kc.L - 1;
+    lidx[j] = min(max(g.ln - (g.d < 0.0 ? 1 : 0), 0), kc.L - 2);
+  }
+  if (exc) {
+    double u_l[N], a_l[N], d_l[N], t_l[N], f_o[N], t_o[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      u_l[j] = u0[j];
+      a_l[j] = acc[j];
+      d_l[j] = dem[j];
+      t_l[j] = thr_max[j];
+    }
+    plant_generic_ool<N>(P.k_dev, S, P.inv_S, P.grid, u_l, a_l, d_l, t_l, f_o, t_o);
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      acc[j] = a_l[j];
+      fbar[j] = f_o[j];
+      thr[j] = t_o[j];
+    }
+    return;
+  }
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    const KnobConst &kc = P.k[j];
+    const PairEntry *e = P.pair + kc.cls * kMaxL + lidx[j];
+    const double2 e0 = __ldg(reinterpret_cast<const double2 *>(&e->mid));
+    const double2 e1 = __ldg(reinterpret_cast<const double2 *>(&e->lev1));
+    const double g1v = __ldg(&e->g1);
+    const double d = dem[j], tm = thr_max[j];
+    const double k0 = __dmul_rn(tm, e1.y), k1 = __dmul_rn(tm, g1v);
+    pair_substeps<S>(u0[j], acc[j], e0.x, e0.y, e1.x, d < k0 ? d : k0, d < k1 ? d : k1, P.inv_S, fbar[j], thr[j]);
+  }
 }
 
 // Trace of the level indices (traced instances only): replays the same

@@ -12,7 +12,7 @@ pytestmark = pytest.mark.gpu
 
 
 @pytest.mark.parametrize("n_gpus,P,M,W", [(3, 8, 2, 2e-4), (2, 8, 3, 5e-4), (1, 6, 4, 1e-4), (4, 8, 2, 3e-3),
-                                          (1, 8, 1, 2e-4)])
+                                          (1, 8, 1, 2e-4), (8, 8, 3, 2e-4), (8, 8, 3, 2e-3), (5, 8, 4, 5e-4)])
 def test_move_closed_loop_parity(G, oracle_mod, n_gpus, P, M, W):
     d = configs.move_suppression(n_servers=160, periods=300, wmove=W, n_gpus=n_gpus, P=P, M=M)
     g, gp, ref = _sim_compare(G, oracle_mod, d, 160, np.array([0, 33, 159]), periods=300)
@@ -28,7 +28,22 @@ def test_move_chunked(G, oracle_mod):
     _sim_compare(G, oracle_mod, d, 64, np.array([0, 63]), periods=150, chunks=[50, 50, 50])
 
 
+def test_move_survey_scale_kkt(G, oracle_mod):
+    """SURVEY §8(f) NEXT-3 at its scale: the 1 CPU + 8 GPU server with M = 3
+    (27 coupled variables; 3^27 brute force is out of reach): the structured
+    active set's u against the oracle's dense generic active set element by
+    element over a closed loop, bound feasibility every period, and no
+    solver-cap status."""
+    d = configs.move_suppression(n_servers=256, periods=200, wmove=5e-4, n_gpus=8, P=8, M=3)
+    g, gp, ref = _sim_compare(G, oracle_mod, d, 256, np.array([0, 100, 255]), periods=200)
+    assert np.all(gp["tr_status"] & G.ST_SOLVER_CAP == 0)
+    lo = np.array([k["f_min"] for k in d["knobs"]]); hi = np.array([k["f_max"] for k in d["knobs"]])
+    u = gp["tr_u"]  # [K][M][N][n_trace]
+    assert np.all(u >= lo[None, None, :, None]) and np.all(u <= hi[None, None, :, None])
+
+
 def test_move_unsupported_shapes(G):
-    d = configs.move_suppression(n_servers=8, n_gpus=8, M=3)
+    """Stacks beyond M N = 36 (e.g. 1 CPU + 15 GPUs at M = 4: 64 variables) are rejected at create."""
+    d = configs.move_suppression(n_servers=8, n_gpus=15, M=4)
     with pytest.raises(G.CapGPUError, match="unsupported"):
         G.CapGPU.from_config(d)
