@@ -14,8 +14,15 @@ demand and throughput-driven weights) - see DESIGN.md §8 for why cfg 3.
 Timing: W untimed warm-up steps, then K timed steps, each bracketed by CUDA
 events on the launching stream; L2 is flushed (256 MiB write) between timed
 steps outside the events; barrier + synchronize on both sides; max over ranks.
-Multi-GPU (torchrun): one process per GPU, weak scaling (each rank runs its own
-disjoint shard of the config, no data-path collective).
+Multi-GPU (torchrun): one process per GPU.  Strong scaling:
+the SAME global problem is split into contiguous 1024-server shards
+(capgpu_shard_range); cfgs 1-3, 5 need no data-path collective (servers are
+independent), cfg 4 all-reduces its 16 KB block vector per period over NCCL.
+`--scaling weak` gives every rank its own full copy of the config instead.
+
+`--call control_step` times the per-period C-ABI call a deployment makes on
+host measurements (capgpu_control_step: S1-S3 on user data, state in HBM):
+HBM roofline; e2e includes the H2D of the measurements and the D2H of u.
 """
 from __future__ import annotations
 
@@ -176,6 +183,113 @@ def oracle_rate(cfg: int, periods: int, budget_s: float, cores: int, single: dic
     return steps / wall, f"{cores * k} instances (strided over the {n_inst}) x {periods} periods", cores, wall
 
 
+# ---------------------------------------------------------------- control_step (per-period call)
+
+def control_step_bytes(N: int, M: int) -> int:
+    """Algorithmic HBM bytes of one capgpu_control_step instance-step: inputs
+    p, cap, f (N), thr (N), thr_max (N) read; the model state (w, mu_p, mu_f,
+    Sigma_ff, Sigma_fp) read + written; A0 read; the warm starts (s_prev, act)
+    read + written; outputs u (M N), active codes (M), status written."""
+    T = N * (N + 1) // 2
+    inputs = 8 * (2 + 3 * N)
+    state = 2 * 8 * (2 + N + T + N) + 8 * N + 2 * 12 * M
+    outputs = 8 * M * N + 4 * M + 4
+    return inputs + state + outputs
+
+
+def bench_control_step(args, d, g, world, rank, local, dev, n_global):
+    """One step = one capgpu_control_step call over every local instance (S1-S3
+    on user measurements): the per-period call of a deployment."""
+    import torch
+    import torch.distributed as dist
+    N, M = d["n_gpus"] + 1, d["M"]
+    n = g.n_inst
+    gen = torch.Generator(device="cpu").manual_seed(7)
+    lo = torch.tensor([k["f_min"] for k in d["knobs"]], dtype=torch.float64)
+    hi = torch.tensor([k["f_max"] for k in d["knobs"]], dtype=torch.float64)
+    f = (lo[:, None] + (hi - lo)[:, None] * torch.rand(N, n, generator=gen, dtype=torch.float64))
+    thr_max = 40 + 160 * torch.rand(N, n, generator=gen, dtype=torch.float64)
+    thr = thr_max * torch.rand(N, n, generator=gen, dtype=torch.float64)
+    p = 600 + 400 * torch.rand(n, generator=gen, dtype=torch.float64)
+    cap = 700 + 300 * torch.rand(n, generator=gen, dtype=torch.float64)
+    host = {k: v.pin_memory() for k, v in dict(p=p, f=f, thr=thr, thr_max=thr_max, cap=cap).items()}
+    devb = {k: v.to(dev) for k, v in host.items()}
+    g.identify()
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+        torch.cuda.synchronize()
+
+    obuf = g.control_step_buffers(ranks=False, ahat=False)  # the controller's outputs: u, codes, status
+    for _ in range(args.warmup):
+        g.control_step(devb["p"], devb["f"], devb["thr"], devb["thr_max"], devb["cap"], out=obuf)
+    barrier()
+    sampler = ClockSampler(local)
+    sampler.start()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    barrier()
+    t0 = time.monotonic()
+    for i in range(args.steps):
+        flush.zero_()
+        evs[i][0].record(stream)
+        g.control_step(devb["p"], devb["f"], devb["thr"], devb["thr_max"], devb["cap"], out=obuf)
+        evs[i][1].record(stream)
+    barrier()
+    clocks = sampler.summary(t0, time.monotonic())
+    t_local = sum(a.elapsed_time(b) for a, b in evs) / 1e3
+    tt = torch.tensor([t_local], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    t_max = float(tt.item())
+    total = n_global * d["workload"]["n_caps"] if args.scaling == "strong" else world * n
+    value = total * args.steps / t_max
+    # e2e: H2D of the period's measurements from pinned host memory, the call,
+    # D2H of the applied frequencies u_0 (what the actuators need)
+    u_host = torch.empty(N, n, dtype=torch.float64, pin_memory=True)
+    e2e = []
+    for _ in range(max(3, args.steps // 2)):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for k in devb:
+            devb[k].copy_(host[k], non_blocking=True)
+        out = g.control_step(devb["p"], devb["f"], devb["thr"], devb["thr_max"], devb["cap"], out=obuf)
+        u_host.copy_(out["u"][0], non_blocking=True)
+        b.record(stream)
+        e2e.append((a, b))
+    barrier()
+    te = torch.tensor([sum(a.elapsed_time(b) for a, b in e2e) / 1e3], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_value = total * len(e2e) / float(te.item())
+    bps = control_step_bytes(N, M)
+    achieved = bps * n / (t_local / args.steps) / 1e9
+    peak = measured_hbm_gbs()
+    if rank == 0:
+        line = {"metric": "server-control-steps/sec", "value": value, "unit": "server-control-steps/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_max / args.steps,
+                "higher_is_better": True, "scaling": "strong" if args.scaling == "strong" else "weak",
+                "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic measurements (seeded uniform p, cap, f, thr within the box)",
+                "config": {"workload": f"capgpu_control_step at the cfg{d['cfg']} shape: {n_global:,} servers, "
+                                       f"N={N}, P/M={d['P']}/{M} (S1-S3 per call, state in HBM)",
+                           "instances_per_gpu": n, "mode": "per-period C-ABI call k_control_step (1 launch per step)",
+                           "l2": "flushed between timed steps (256 MiB write outside the events)",
+                           "parallelism": f"dp{world}"},
+                "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                             "frac": achieved / peak, "traffic": None, "bytes_per_step": bps,
+                             "peak_source": "MEASURED_PEAKS.json hbm_gbs"},
+                "e2e": {"value": e2e_value, "unit": "server-control-steps/s",
+                        "h2d_bytes_per_step": 8 * n * (2 + 3 * N), "d2h_bytes_per_step": 8 * n * N},
+                "gpu_launches": args.steps, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
 # ---------------------------------------------------------------- main
 
 def parse():
@@ -188,6 +302,9 @@ def parse():
     ap.add_argument("--impl", default="capgpu", choices=["capgpu", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle work for cpu_baseline")
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="multi-GPU: split one global problem (strong, SURVEY §8(d.1)) or replicate it (weak)")
+    ap.add_argument("--call", default="simulate", choices=["simulate", "control_step"])
     return ap.parse_args()
 
 
@@ -267,13 +384,21 @@ def main():
             nccl_id = bytes(uid.cpu().tolist())
         g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=begin, world=world, rank=rank,
                                n_servers_global=n_global, nccl_id=nccl_id)
+    elif args.scaling == "strong":
+        # cfgs 1-3, 5: independent servers; the global problem is split into
+        # contiguous 1024-aligned shards, no data-path collective
+        n_global = d["n_servers"]
+        begin, n_srv = G.shard_range(n_global, world, rank, 1024 if n_global >= 1024 * world else 1)
+        g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=begin, world=world, rank=rank,
+                               n_servers_global=n_global)
     else:
-        # cfgs 1-3, 5: independent servers; every rank runs its own shard of the
-        # configuration (weak scaling, no data-path collective)
+        # weak scaling: every rank runs its own disjoint copy of the configuration
         n_srv = d["n_servers"]
         n_global = world * n_srv
         g = CapGPU.from_config(d, n_servers=n_srv, srv_begin=rank * n_srv, world=world, rank=rank,
                                n_servers_global=n_global)
+    if args.call == "control_step":
+        return bench_control_step(args, d, g, world, rank, local, dev, n_global)
     wl = workload_from(d)
     n_inst = g.n_inst
     stream = torch.cuda.current_stream()
@@ -310,7 +435,8 @@ def main():
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     t_max = float(tt.item())
     steps_per_call = n_inst * periods
-    total_per_step = (n_global if hier else world * n_inst) * periods
+    caps = d["workload"]["n_caps"]
+    total_per_step = (n_global if hier else (n_global * caps if args.scaling == "strong" else world * n_inst)) * periods
     value = total_per_step * args.steps / t_max
 
     # ---- e2e through the public API with host buffers: H2D of the per-instance
@@ -389,18 +515,22 @@ def main():
                     "state_bytes_per_step": state_bytes_per_instance(N, M) / periods}
             mode = ("fused multi-period kernel k_simulate (1 launch per step)" if ctrl == 0 else
                     "fused multi-period baseline kernel k_baseline (1 launch per step)")
-            par = f"dp{world} (server shards, no data-path collective)"
+            par = (f"dp{world} ({'strong: the global problem in contiguous 1024-server shards'
+                                if args.scaling == 'strong' else 'weak: one full copy per rank'}, "
+                   "no data-path collective)")
             launches = args.steps
         if ncu_pipe:
             roof["ncu"] = ncu_pipe
         line = {"metric": "server-control-steps/sec", "value": value, "unit": "server-control-steps/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": 1e3 * t_max / args.steps, "higher_is_better": True,
-                "scaling": "strong" if hier else "weak",
+                "scaling": "strong" if (hier or args.scaling == "strong") else "weak",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded generator, DESIGN.md §3)",
                 "config": {"workload": workload_name(d, periods), "instances_per_gpu": n_inst,
                            "periods_per_step": periods, "n_knobs": N, "P": d["P"], "M": M, "substeps": S,
                            "mode": mode,
+                           "global_instances": (n_global * caps if not hier else n_global),
+                           "per_period_us": 1e6 * t_max / args.steps / periods,
                            "l2": "flushed between timed steps (256 MiB write outside the events)",
                            "parallelism": par},
                 "roofline": roof,

@@ -271,6 +271,28 @@ int capgpu_tree_sum_host(const double *v, int64_t n, double *out);
 int capgpu_sim_state(capgpu_ctx *ctx, double *fbar_d, double *acc_d, double *thr_d, double *p_d,
                      void *stream);
 
+/* Overwrite the plant state of the simulation (inverse of capgpu_sim_state;
+ * device pointers, each nullable = keep).  Validated before anything is
+ * written (synchronous on `stream`): every value finite and |acc_j| <=
+ * step_j / 2 -- the first-order modulator's invariant (Q15) that the
+ * plant's exactness rests on; else CAPGPU_E_INVALID and nothing changes.
+ * CAPGPU_E_ORDER before the first capgpu_simulate. */
+int capgpu_set_state(capgpu_ctx *ctx, const double *fbar_d, const double *acc_d, const double *thr_d,
+                     const double *p_d, void *stream);
+
+/* Checkpoint / resume of a whole context: the model state (S1),
+ * plant state (S4), warm starts (S3), server constants, the period counter and
+ * -- for the hierarchical budget -- the per-server weights and cluster
+ * aggregates, as one device blob of capgpu_checkpoint_bytes(ctx) bytes
+ * (caller-owned, e.g. a torch uint8 tensor; copy it to the host to persist).
+ * Load into a context created with the SAME arguments (checked: else
+ * CAPGPU_E_INVALID); a hierarchical checkpoint needs the budget allocated
+ * first (one simulate call, else CAPGPU_E_ORDER).  A resumed run continues
+ * bitwise identically.  save/load synchronise `stream`. */
+int64_t capgpu_checkpoint_bytes(const capgpu_ctx *ctx);
+int capgpu_checkpoint_save(capgpu_ctx *ctx, void *dst_d, void *stream);
+int capgpu_checkpoint_load(capgpu_ctx *ctx, const void *src_d, void *stream);
+
 /* Current base caps P_s of every local instance (device [n_inst], W); valid
  * after the first capgpu_simulate. */
 int capgpu_sim_caps(capgpu_ctx *ctx, double *cap_base_d, void *stream);

@@ -78,7 +78,8 @@ SYMBOLS = ["capgpu_version", "capgpu_status_string", "capgpu_last_error", "capgp
            "capgpu_model_reset", "capgpu_assign_weights", "capgpu_control_step", "capgpu_simulate",
            "capgpu_sim_reset", "capgpu_sim_state", "capgpu_sim_caps", "capgpu_nccl_unique_id", "capgpu_shard_range",
            "capgpu_debug_gen", "capgpu_fp64_peak", "capgpu_simulate_group", "capgpu_tree_sum_host",
-           "capgpu_debug_phase_counters"]
+           "capgpu_debug_phase_counters", "capgpu_set_state", "capgpu_checkpoint_bytes", "capgpu_checkpoint_save",
+           "capgpu_checkpoint_load"]
 
 _lib = None
 
@@ -116,6 +117,11 @@ def lib():
     L.capgpu_sim_reset.argtypes = [_VP]
     L.capgpu_sim_state.argtypes = [_VP, _VP, _VP, _VP, _VP, _VP]
     L.capgpu_sim_caps.argtypes = [_VP, _VP, _VP]
+    L.capgpu_set_state.argtypes = [_VP, _VP, _VP, _VP, _VP, _VP]
+    L.capgpu_checkpoint_bytes.argtypes = [_VP]
+    L.capgpu_checkpoint_bytes.restype = C.c_int64
+    L.capgpu_checkpoint_save.argtypes = [_VP, _VP, _VP]
+    L.capgpu_checkpoint_load.argtypes = [_VP, _VP, _VP]
     L.capgpu_nccl_unique_id.argtypes = [C.POINTER(C.c_uint8 * 128)]
     L.capgpu_shard_range.argtypes = [C.c_int64, C.c_int32, C.c_int32, C.c_int64, C.POINTER(C.c_int64)]
     L.capgpu_shard_range.restype = C.c_int64
@@ -307,17 +313,21 @@ class CapGPU:
         return th, R, rk
 
     # ---- S1-S3 on user measurements
-    def control_step(self, p_meas, f_applied, thr, thr_max, cap):
+    def control_step_buffers(self, ranks: bool = True, ahat: bool = True):
+        """Output buffers of control_step (written entirely by the kernel; reusable)."""
         n = self.n_srv
-        u = self._z(self.M, self.N, n)
-        act = self._z(self.M, n, dtype=torch.int32)
-        rk = self._z(self.N, n, dtype=torch.int8)
-        ah = self._z(self.N, n)
-        st = self._z(n, dtype=torch.int32)
+        return dict(u=self._z(self.M, self.N, n), active=self._z(self.M, n, dtype=torch.int32),
+                    rank=self._z(self.N, n, dtype=torch.int8) if ranks else None,
+                    ahat=self._z(self.N, n) if ahat else None, status=self._z(n, dtype=torch.int32))
+
+    def control_step(self, p_meas, f_applied, thr, thr_max, cap, out=None):
+        o = out if out is not None else self.control_step_buffers()
+        opt = lambda t: _ptr(t) if t is not None else None  # noqa: E731
         _check(self.L.capgpu_control_step(self._ctx, _ptr(p_meas), _ptr(f_applied), _ptr(thr), _ptr(thr_max),
-                                          _ptr(cap), _ptr(u), _ptr(act), _ptr(rk), _ptr(ah), _ptr(st), _stream()),
+                                          _ptr(cap), _ptr(o["u"]), _ptr(o["active"]), opt(o["rank"]),
+                                          opt(o["ahat"]), _ptr(o["status"]), _stream()),
                self._ctx)
-        return dict(u=u, active=act, rank=rk, ahat=ah, status=st)
+        return o
 
     # ---- closed loop
     def summary_buffers(self):
@@ -373,6 +383,19 @@ class CapGPU:
         f, a, t, p = self._z(N, ni), self._z(N, ni), self._z(N, ni), self._z(ni)
         _check(self.L.capgpu_sim_state(self._ctx, _ptr(f), _ptr(a), _ptr(t), _ptr(p), _stream()), self._ctx)
         return dict(fbar=f, acc=a, thr=t, p=p)
+
+    def set_state(self, fbar=None, acc=None, thr=None, p=None):
+        _check(self.L.capgpu_set_state(self._ctx, _ptr(fbar), _ptr(acc), _ptr(thr), _ptr(p), _stream()), self._ctx)
+
+    def checkpoint(self):
+        """Device blob (torch uint8) holding the whole context state (checkpoint / resume)."""
+        buf = torch.empty(int(self.L.capgpu_checkpoint_bytes(self._ctx)), dtype=torch.uint8, device="cuda")
+        _check(self.L.capgpu_checkpoint_save(self._ctx, _ptr(buf), _stream()), self._ctx)
+        return buf
+
+    def restore(self, blob):
+        blob = blob.to("cuda")
+        _check(self.L.capgpu_checkpoint_load(self._ctx, _ptr(blob), _stream()), self._ctx)
 
     def sim_caps(self):
         out = self._z(self.n_inst)

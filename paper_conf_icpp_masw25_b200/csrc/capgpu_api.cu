@@ -847,20 +847,21 @@ int capgpu_simulate_group(capgpu_ctx **ctxs, int32_t n_ctx, int64_t periods, con
   Budget *bs[64];
   for (int q = 0; q < n_ctx; ++q) bs[q] = &ctxs[q]->budget;
   const int64_t k0 = ctxs[0]->k_global;
-  for (int64_t kk = 0; kk < periods; ++kk) {
-    for (int q = 0; q < n_ctx; ++q) {
-      capgpu_ctx *c = ctxs[q];
-      int rc = budget_period_local(c->budget, c->dp, c->st, t[q], c->L, k0 + kk, (int)kk, (int)periods, s, c->err);
-      if (rc) return rc;
-    }
-    int rc = budget_reduce(bs, n_ctx, false, s, ctxs[0]->err);
+  DevParams Ps[64];
+  StatePtrs Ss[64];
+  Launchers Ls[64];
+  double *aW[64], *aP[64];
+  for (int q = 0; q < n_ctx; ++q) {
+    Ps[q] = ctxs[q]->dp;
+    Ss[q] = ctxs[q]->st;
+    Ls[q] = ctxs[q]->L;
+    const capgpu_trace *tq = trs ? trs[q] : nullptr;
+    aW[q] = tq ? tq->agg_W_d : nullptr;
+    aP[q] = tq ? tq->agg_P_d : nullptr;
+  }
+  {
+    int rc = budget_simulate_group(bs, n_ctx, Ps, Ss, t, Ls, k0, periods, aW, aP, s, ctxs[0]->err);
     if (rc) return rc;
-    for (int q = 0; q < n_ctx; ++q) {
-      const capgpu_trace *tq = trs ? trs[q] : nullptr;
-      rc = budget_tree(ctxs[q]->budget, tq ? tq->agg_W_d : nullptr, tq ? tq->agg_P_d : nullptr, (int)kk, s,
-                       ctxs[q]->err);
-      if (rc) return rc;
-    }
   }
   for (int q = 0; q < n_ctx; ++q) ctxs[q]->k_global += periods;
   return CAPGPU_OK;
@@ -878,6 +879,154 @@ int capgpu_sim_state(capgpu_ctx *c, double *fbar_d, double *acc_d, double *thr_d
   if (acc_d) CK_CUDA(c, cudaMemcpyAsync(acc_d, c->st.acc, nb, cudaMemcpyDeviceToDevice, s));
   if (thr_d) CK_CUDA(c, cudaMemcpyAsync(thr_d, c->st.thr, nb, cudaMemcpyDeviceToDevice, s));
   if (p_d) CK_CUDA(c, cudaMemcpyAsync(p_d, c->st.p, sizeof(double) * c->n_inst, cudaMemcpyDeviceToDevice, s));
+  return CAPGPU_OK;
+}
+
+// ---- state setter and checkpoint / resume
+
+// |acc_j| <= step_j / 2 (+ rounding) is the modulator invariant the plant relies
+// on (plant_pair); flags violations of a candidate acc array
+__global__ void k_check_acc(const double *acc, int64_t n, const KnobConst *k, int N, int *bad) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  for (int j = 0; j < N; ++j) {
+    const double a = acc[(int64_t)j * n + i];
+    if (!(fabs(a) <= 0.5 * k[j].step * (1.0 + 1e-9))) atomicOr(bad, 1);
+  }
+}
+__global__ void k_check_finite(const double *x, int64_t n, int *bad) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n && !isfinite(x[i])) atomicOr(bad, 2);
+}
+
+int capgpu_set_state(capgpu_ctx *c, const double *fbar_d, const double *acc_d, const double *thr_d,
+                     const double *p_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  if (!c->sim_ready) return fail(c, CAPGPU_E_ORDER, "simulation not initialised (call capgpu_simulate first)");
+  OPT_DEV(c, fbar_d);
+  OPT_DEV(c, acc_d);
+  OPT_DEV(c, thr_d);
+  OPT_DEV(c, p_d);
+  cudaStream_t s = (cudaStream_t)stream;
+  const int64_t nn = (int64_t)c->N * c->n_inst;
+  // validation before anything is written: finite values, |acc| <= step / 2
+  int *bad = nullptr;
+  CK_CUDA(c, cudaMalloc(&bad, sizeof(int)));
+  int hbad = 0;
+  cudaError_t e = cudaMemsetAsync(bad, 0, sizeof(int), s);
+  const double *arrs[4] = {fbar_d, acc_d, thr_d, p_d};
+  const int64_t lens[4] = {nn, nn, nn, c->n_inst};
+  for (int q = 0; q < 4 && e == cudaSuccess; ++q)
+    if (arrs[q]) {
+      k_check_finite<<<grid_for(lens[q], 256), 256, 0, s>>>(arrs[q], lens[q], bad);
+      e = cudaGetLastError();
+    }
+  if (e == cudaSuccess && acc_d) {
+    k_check_acc<<<grid_for(c->n_inst, 256), 256, 0, s>>>(acc_d, c->n_inst, c->dp.k_dev, c->N, bad);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaFree(bad);
+  if (e != cudaSuccess) return cuda_fail(c, e, "set_state validation");
+  if (hbad & 2) return fail(c, CAPGPU_E_INVALID, "set_state: non-finite value");
+  if (hbad & 1) return fail(c, CAPGPU_E_INVALID, "set_state: |acc| exceeds half a grid step (modulator invariant)");
+  const size_t nb = sizeof(double) * (size_t)nn;
+  if (fbar_d) CK_CUDA(c, cudaMemcpyAsync(c->st.fbar, fbar_d, nb, cudaMemcpyDeviceToDevice, s));
+  if (acc_d) CK_CUDA(c, cudaMemcpyAsync(c->st.acc, acc_d, nb, cudaMemcpyDeviceToDevice, s));
+  if (thr_d) CK_CUDA(c, cudaMemcpyAsync(c->st.thr, thr_d, nb, cudaMemcpyDeviceToDevice, s));
+  if (p_d) CK_CUDA(c, cudaMemcpyAsync(c->st.p, p_d, sizeof(double) * c->n_inst, cudaMemcpyDeviceToDevice, s));
+  return CAPGPU_OK;
+}
+
+// Checkpoint blob: a fixed header, the whole state workspace (model, plant,
+// warm starts, server constants, grid tables -- identical for identical
+// create() arguments), and for the hierarchical budget its per-server weights
+// and cluster aggregates.
+namespace {
+struct CkptHeader {
+  uint64_t magic;
+  int64_t n_srv, n_inst, ws_bytes, k_global, budget_doubles;
+  int32_t N, M, P, flags;
+  capgpu_workload wl;
+  double B_c, pmin_tot, pmax_tot;
+};
+constexpr uint64_t kCkptMagic = 0x3150434B55504743ull;  // "CGPUKCP1"
+int64_t budget_doubles(const capgpu_ctx *c) { return c->budget.ready ? c->n_srv + 4 : 0; }
+}  // namespace
+
+int64_t capgpu_checkpoint_bytes(const capgpu_ctx *c) {
+  if (!c) return 0;
+  const int64_t hb = ((int64_t)sizeof(CkptHeader) + 255) & ~(int64_t)255;
+  return hb + c->ws_bytes + 8 * budget_doubles(c);
+}
+
+int capgpu_checkpoint_save(capgpu_ctx *c, void *dst_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, dst_d);
+  cudaStream_t s = (cudaStream_t)stream;
+  CkptHeader h{};
+  h.magic = kCkptMagic;
+  h.n_srv = c->n_srv;
+  h.n_inst = c->n_inst;
+  h.ws_bytes = c->ws_bytes;
+  h.k_global = c->k_global;
+  h.budget_doubles = budget_doubles(c);
+  h.N = c->N;
+  h.M = c->M;
+  h.P = c->P;
+  h.flags = (c->servers_ready ? 1 : 0) | (c->has_prior ? 2 : 0) | (c->sim_ready ? 4 : 0) | (c->budget.ready ? 8 : 0);
+  h.wl = c->wl;
+  h.B_c = c->budget.B_c;
+  h.pmin_tot = c->budget.pmin_tot;
+  h.pmax_tot = c->budget.pmax_tot;
+  const int64_t hb = ((int64_t)sizeof(CkptHeader) + 255) & ~(int64_t)255;
+  char *d = (char *)dst_d;
+  CK_CUDA(c, cudaMemcpyAsync(d + hb, c->ws, (size_t)c->ws_bytes, cudaMemcpyDeviceToDevice, s));
+  if (h.budget_doubles) {
+    double *bd = (double *)(d + hb + c->ws_bytes);
+    CK_CUDA(c, cudaMemcpyAsync(bd, c->budget.srv_w, sizeof(double) * c->n_srv, cudaMemcpyDeviceToDevice, s));
+    CK_CUDA(c, cudaMemcpyAsync(bd + c->n_srv, c->budget.agg, sizeof(double) * 2, cudaMemcpyDeviceToDevice, s));
+    CK_CUDA(c, cudaMemcpyAsync(bd + c->n_srv + 2, c->budget.consts, sizeof(double) * 2, cudaMemcpyDeviceToDevice, s));
+  }
+  // the header comes from host memory: synchronous, so h may go out of scope
+  CK_CUDA(c, cudaStreamSynchronize(s));
+  CK_CUDA(c, cudaMemcpy(d, &h, sizeof h, cudaMemcpyHostToDevice));
+  return CAPGPU_OK;
+}
+
+int capgpu_checkpoint_load(capgpu_ctx *c, const void *src_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, src_d);
+  cudaStream_t s = (cudaStream_t)stream;
+  CkptHeader h{};
+  CK_CUDA(c, cudaStreamSynchronize(s));
+  CK_CUDA(c, cudaMemcpy(&h, src_d, sizeof h, cudaMemcpyDeviceToHost));
+  if (h.magic != kCkptMagic) return fail(c, CAPGPU_E_INVALID, "checkpoint: bad magic");
+  if (h.n_srv != c->n_srv || h.n_inst != c->n_inst || h.ws_bytes != c->ws_bytes || h.N != c->N || h.M != c->M ||
+      h.P != c->P)
+    return fail(c, CAPGPU_E_INVALID, "checkpoint: shape differs from this context (create it with the same arguments)");
+  if ((h.flags & 8) && !c->budget.srv_w)
+    return fail(c, CAPGPU_E_ORDER, "checkpoint holds a hierarchical budget: run one capgpu_simulate with the "
+                                   "hierarchical workload (or simulate_group) before loading");
+  const int64_t hb = ((int64_t)sizeof(CkptHeader) + 255) & ~(int64_t)255;
+  const char *d = (const char *)src_d;
+  CK_CUDA(c, cudaMemcpyAsync(c->ws, d + hb, (size_t)c->ws_bytes, cudaMemcpyDeviceToDevice, s));
+  if (h.budget_doubles) {
+    const double *bd = (const double *)(d + hb + c->ws_bytes);
+    CK_CUDA(c, cudaMemcpyAsync(c->budget.srv_w, bd, sizeof(double) * c->n_srv, cudaMemcpyDeviceToDevice, s));
+    CK_CUDA(c, cudaMemcpyAsync(c->budget.agg, bd + c->n_srv, sizeof(double) * 2, cudaMemcpyDeviceToDevice, s));
+    CK_CUDA(c, cudaMemcpyAsync(c->budget.consts, bd + c->n_srv + 2, sizeof(double) * 2, cudaMemcpyDeviceToDevice, s));
+    c->budget.B_c = h.B_c;
+    c->budget.pmin_tot = h.pmin_tot;
+    c->budget.pmax_tot = h.pmax_tot;
+    c->budget.ready = true;
+  }
+  c->servers_ready = h.flags & 1;
+  c->has_prior = (h.flags & 2) != 0;
+  c->sim_ready = (h.flags & 4) != 0;
+  c->k_global = h.k_global;
+  c->wl = h.wl;
   return CAPGPU_OK;
 }
 

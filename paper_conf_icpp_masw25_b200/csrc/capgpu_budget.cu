@@ -8,7 +8,10 @@
 // the cluster sum is a fixed pairwise tree over the padded block vector.  The
 // result is bitwise identical on every GPU and for 1, 2, 4 or 8 GPUs.
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
+
+#define CAPGPU_UNUSED(x) (void)(x)
 
 #include <nccl.h>
 
@@ -37,7 +40,8 @@ __global__ void k_block_sums(const double *part, int64_t n_cta, int64_t nb_local
 // for h = len/2 .. 1: v[i] += v[i + h], i < h.  Same order as
 // capgpu_tree_sum_host.  Single CTA; two vectors (w, p) side by side.
 __global__ void k_tree(const double *recv, int64_t nb_g, int64_t len, double *scratch, double *agg, double *tW,
-                       double *tP, int kk) {
+                       double *tP, int kk, int64_t *kdev) {
+  if (kdev) kk = (int)kdev[1];  // graph replay: call period from device memory, advanced below
   for (int64_t i = threadIdx.x; i < len; i += blockDim.x) {
     scratch[i] = i < nb_g ? recv[i] : 0.0;
     scratch[len + i] = i < nb_g ? recv[nb_g + i] : 0.0;
@@ -55,7 +59,13 @@ __global__ void k_tree(const double *recv, int64_t nb_g, int64_t len, double *sc
     agg[1] = scratch[len];
     if (tW) tW[kk] = scratch[0];
     if (tP) tP[kk] = scratch[len];
+    if (kdev) kdev[1] = kk + 1;  // every thread read kdev[1] before the first __syncthreads
   }
+}
+
+__global__ void k_set_period(int64_t *kdev, int64_t k0) {
+  kdev[0] = k0;
+  kdev[1] = 0;
 }
 
 __global__ void k_accumulate(double *dst, const double *src, int64_t n, int first) {
@@ -72,6 +82,7 @@ static BudgetDev dev_view(Budget &b) {
   d.pmin_tot = b.pmin_tot;
   d.rack_frac = b.rack_frac;
   d.rack = b.rack;
+  d.kdev = b.graph_mode ? b.kdev : nullptr;
   return d;
 }
 
@@ -106,6 +117,8 @@ void budget_free(Budget &b) {
   for (double *p : bufs)
     if (p) cudaFree(p);
   b.srv_w = b.part = b.part_c = b.send = b.recv = b.scratch = b.agg = b.consts = nullptr;
+  if (b.kdev) cudaFree(b.kdev);
+  b.kdev = nullptr;
   b.ready = false;
 }
 
@@ -151,6 +164,7 @@ int budget_alloc(Budget &b, const DevParams &P, const capgpu_workload &wl, const
   BCK(cudaMalloc(&b.scratch, sizeof(double) * 2 * b.tree_len));
   BCK(cudaMalloc(&b.agg, sizeof(double) * 2));
   BCK(cudaMalloc(&b.consts, sizeof(double) * 2));
+  BCK(cudaMalloc(&b.kdev, sizeof(int64_t) * 2));
   BCK(cudaMemset(b.send, 0, sizeof(double) * 2 * b.nb_g));
   BCK(cudaMemset(b.recv, 0, sizeof(double) * 2 * b.nb_g));
   return CAPGPU_OK;
@@ -204,7 +218,8 @@ int budget_reduce(Budget **bs, int n, bool /*consts*/, cudaStream_t s, char *err
 }
 
 int budget_tree(Budget &b, double *agg_W, double *agg_P, int kk, cudaStream_t s, char *err) {
-  k_tree<<<1, 1024, 0, s>>>(b.recv, b.nb_g, b.tree_len, b.scratch, b.agg, agg_W, agg_P, kk);
+  k_tree<<<1, 1024, 0, s>>>(b.recv, b.nb_g, b.tree_len, b.scratch, b.agg, agg_W, agg_P, kk,
+                            b.graph_mode ? b.kdev : nullptr);
   BCK(cudaGetLastError());
   return CAPGPU_OK;
 }
@@ -240,11 +255,78 @@ int budget_period_local(Budget &b, const DevParams &P, const StatePtrs &st, cons
 int budget_simulate(Budget &b, const DevParams &P, const StatePtrs &st, const TracePtrs &tr, const Launchers &L,
                     int64_t k0, int64_t K, double *agg_W, double *agg_P, cudaStream_t s, char *err) {
   Budget *bs[1] = {&b};
-  for (int64_t kk = 0; kk < K; ++kk) {
-    int rc = budget_period_local(b, P, st, tr, L, k0 + kk, (int)kk, (int)K, s, err);
-    if (!rc) rc = budget_reduce(bs, 1, false, s, err);
-    if (!rc) rc = budget_tree(b, agg_W, agg_P, (int)kk, s, err);
+  CAPGPU_UNUSED(bs);
+  return budget_simulate_group(bs, 1, &P, &st, &tr, &L, k0, K, agg_W ? &agg_W : nullptr, agg_P ? &agg_P : nullptr, s,
+                               err);
+}
+
+// The K periods of a call for n budgets (1 = one context on its GPU, NCCL if
+// world > 1; n > 1 = loopback shards of one GPU).  One period = k_period +
+// block sums of every context, the all-reduce, every context's tree.  With
+// CUDA-graph replay (default for K >= 8; env CAPGPU_NO_GRAPH=1 disables) the
+// period's launches are captured once (R periods unrolled, R <= 16) with the
+// period index read from device memory (k_set_period / k_tree), and the
+// graph is replayed: no per-period host launch gaps.  Same kernels, same
+// order: bitwise identical results.
+int budget_simulate_group(Budget **bs, int n, const DevParams *P, const StatePtrs *st, const TracePtrs *tr,
+                          const Launchers *L, int64_t k0, int64_t K, double **agg_W, double **agg_P, cudaStream_t s,
+                          char *err) {
+  auto period = [&](int64_t kk) -> int {
+    for (int q = 0; q < n; ++q) {
+      int rc = budget_period_local(*bs[q], P[q], st[q], tr[q], L[q], k0 + kk, (int)kk, (int)K, s, err);
+      if (rc) return rc;
+    }
+    int rc = budget_reduce(bs, n, false, s, err);
     if (rc) return rc;
+    for (int q = 0; q < n; ++q) {
+      rc = budget_tree(*bs[q], agg_W ? agg_W[q] : nullptr, agg_P ? agg_P[q] : nullptr, (int)kk, s, err);
+      if (rc) return rc;
+    }
+    return CAPGPU_OK;
+  };
+  const char *ng = getenv("CAPGPU_NO_GRAPH");
+  const bool graph = K >= 8 && !(ng && ng[0] && ng[0] != '0');
+  if (!graph) {
+    for (int64_t kk = 0; kk < K; ++kk) {
+      int rc = period(kk);
+      if (rc) return rc;
+    }
+    return CAPGPU_OK;
+  }
+  for (int q = 0; q < n; ++q) {
+    k_set_period<<<1, 1, 0, s>>>(bs[q]->kdev, k0);
+    BCK(cudaGetLastError());
+    bs[q]->graph_mode = true;
+  }
+  const int R = (int)(K < 16 ? K : 16);
+  cudaStream_t cs;
+  BCK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  int rc = CAPGPU_OK;
+  cudaError_t e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
+  if (e == cudaSuccess) {
+    cudaStream_t s_save = s;
+    s = cs;
+    for (int r = 0; r < R && !rc; ++r) rc = period(r);  // kk in the captured launches is overridden by kdev
+    s = s_save;
+    e = cudaStreamEndCapture(cs, &g);
+  }
+  if (!rc && e == cudaSuccess) e = cudaGraphInstantiate(&ge, g, 0);
+  if (!rc && e == cudaSuccess) {
+    int64_t done = 0;
+    for (; done + R <= K && e == cudaSuccess; done += R) e = cudaGraphLaunch(ge, s);
+    for (int64_t kk = done; kk < K && !rc && e == cudaSuccess; ++kk) rc = period(kk);  // remainder, kdev-driven
+  }
+  for (int q = 0; q < n; ++q) bs[q]->graph_mode = false;
+  if (ge) cudaGraphExecDestroy(ge);
+  if (g) cudaGraphDestroy(g);
+  cudaStreamDestroy(cs);
+  if (rc) return rc;
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    snprintf(err, 512, "period graph: %s", cudaGetErrorString(e));
+    return CAPGPU_E_CUDA;
   }
   return CAPGPU_OK;
 }

@@ -27,6 +27,8 @@ struct Budget {
   double B_c = 0.0, pmin_tot = 0.0, pmax_tot = 0.0, rack_frac = 0.9, cluster_frac = 0.55;
   int rack = 16;
   bool ready = false;
+  int64_t *kdev = nullptr;  // [2] {first period of the call, call period} for CUDA-graph replay
+  bool graph_mode = false;  // launches read the period from kdev (while a call is captured / replayed)
 };
 
 int budget_init_nccl(Budget &b, const uint8_t *id, int world, int rank, char *err);
@@ -43,5 +45,8 @@ int budget_period_local(Budget &b, const DevParams &P, const StatePtrs &st, cons
 int budget_tree(Budget &b, double *agg_W, double *agg_P, int kk, cudaStream_t s, char *err);
 int budget_simulate(Budget &b, const DevParams &P, const StatePtrs &st, const TracePtrs &tr, const Launchers &L,
                     int64_t k0, int64_t K, double *agg_W, double *agg_P, cudaStream_t s, char *err);
+int budget_simulate_group(Budget **bs, int n, const DevParams *P, const StatePtrs *st, const TracePtrs *tr,
+                          const Launchers *L, int64_t k0, int64_t K, double **agg_W, double **agg_P, cudaStream_t s,
+                          char *err);
 
 }  // namespace capgpu

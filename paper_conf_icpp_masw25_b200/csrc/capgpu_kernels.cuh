@@ -1195,6 +1195,8 @@ struct BudgetDev {
   double *cta_part;    // [2][n_cta] this instant's per-CTA partial sums of (w, p)
   double B_c, pmin_tot, rack_frac;
   int32_t rack;        // power of two <= 32
+  const int64_t *kdev; // CUDA-graph replay: {first period of the call, call period} in device memory
+                       // (advanced by k_tree), overriding the k / kk launch parameters; else null
 };
 
 // sum over aligned groups of `g` lanes; commutativity makes every lane of a
@@ -1540,6 +1542,10 @@ __device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs 
 template <int N, int M, int SS>
 __global__ void __launch_bounds__(kPeriodCta, kPeriodWarps * 32 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
                                                 int kk, int K) {
+  if (bd.kdev) {  // graph replay: the period comes from device memory
+    kk = (int)bd.kdev[1];
+    k = bd.kdev[0] + kk;
+  }
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = i < P.n_srv;
   using PT = PeriodTile<N>;
