@@ -106,6 +106,8 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None, v
         return lib
     only = [int(x) for x in os.environ.get("CAPGPU_ONLY_N", "").split(",") if x] if variant else []
     if only:  # experiment build with a subset of the knob counts (smaller library to ship)
+        bdir = bdir + "_n" + "-".join(map(str, sorted(only)))  # objects depend on the subset
+        os.makedirs(bdir, exist_ok=True)
         srcs = [s_ for s_ in srcs if not os.path.basename(s_).startswith("inst_n") or
                 int(os.path.basename(s_)[6:-3]) in only]
         extra = list(extra) + ["-DCAPGPU_SUBSET"] + [

@@ -205,6 +205,10 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   c->shard = sh;
   for (int j = 0; j < N; ++j) c->bounds[j] = bounds[j];
   c->L = launchers(N, h.M);
+  if (!c->L.simulate || !c->L.init_servers) {  // an experiment build without this knob count
+    delete c;
+    return fail(nullptr, CAPGPU_E_UNSUPPORTED, "this library was built without N = %d knobs", N);
+  }
 
   // ---- per-launch constants
   DevParams &d = c->dp;

@@ -523,8 +523,13 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
   // loop body (not unrolled: instruction cache); the per-block registers
   // rotate so the body indexes no array by t.  act[] holds last period's codes
   // on entry (warm start) and this period's on exit.
-  const KnobConst *kc = SLO ? P.k_dev_slo[phase] : P.k;
-  const KnobConst *kc_dev = SLO ? kc : P.k_dev;
+  const KnobConst *kc_src = SLO ? P.k_dev_slo[phase] : P.k;
+  const KnobConst *kc_dev = SLO ? kc_src : P.k_dev;
+  // the instant's bounds in registers (the SLO phases' copies live in global
+  // memory: one read per knob and period instead of one per use)
+  KnobConst kc[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) kc[j] = kc_src[j];
   {
     double smin = 0.0, smax = 0.0;
 #pragma unroll
@@ -535,6 +540,9 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
     status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
     if constexpr (SLO) status |= P.st_slo[phase];
   }
+  // blocks 0 .. M-2 share c = Q (Q11): one problem, solved once (block 0)
+  // unless the reference trajectory gives them different offsets (Q37)
+  const bool shared = !P.ref;
 #pragma unroll 1
   for (int t = 0; t < M; ++t) {
     double ctau[N];
@@ -544,8 +552,33 @@ __device__ __forceinline__ double control_instant(const DevParams &P, double inv
     uint32_t code;
     // Q37: with the reference trajectory block t tracks beta + ref_w[t] (P_s - p(k))
     const double beta_t = P.ref ? fma(P.ref_w[t], cap - p, beta) : beta;
-    const double s = solve_block<N>(kc, kc_dev, ahat, ctau, beta_t, s_prev[0]);
-    code = block_codes<N>(kc, ctau, s);
+    double s;
+    if (t > 0 && t < M - 1 && shared) {
+      s = s_prev[M - 1];  // block t == block 0 (rotated into s_prev[M-1] / act[M-1] last iteration)
+      code = act[M - 1];
+    } else if (t == M - 1 && M > 1 && !out.full && !out.u) {
+      // untraced last block: only "is any bound active at the root" feeds the
+      // summaries; it is iff the all-free root s_f = (beta + A.m) / (1 + sum c tau A)
+      // violates a bound (the unconstrained minimiser is feasible <=> it is the solution)
+      double num = beta_t, den = 1.0;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        num = fma(ahat[j], kc[j].m, num);
+        den = fma(ctau[j], ahat[j], den);
+      }
+      const double sf = num * rcp_fast(den);
+      bool any = false;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        const double v = fma(-ctau[j], sf, kc[j].m);
+        any |= v < kc[j].lo || v > kc[j].hi;
+      }
+      s = sf;
+      code = any ? 2u : 0u;
+    } else {
+      s = solve_block<N>(kc, kc_dev, ahat, ctau, beta_t, s_prev[0]);
+      code = block_codes<N>(kc, ctau, s);
+    }
     if (t == 0 || out.u) {
       double u[N];
       code = block_u<N>(kc, ctau, s, u);
@@ -738,7 +771,6 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
   double p = __ldcg(st.p + i), w = __ldcg(st.w + i), mu_p = __ldcg(st.mu_p + i);
   const double c_true = st.c_true[si], cap_base = st.cap_base[i];
   double s_prev[M];
-#pragma unroll
   uint32_t act[M];
 #pragma unroll
   for (int t = 0; t < M; ++t) {
@@ -1655,11 +1687,18 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
     s_prev[t] = st.s_prev[t * ld + i];
     act[t] = st.act[t * ld + i];
   }
-  const GlobAcc S{st.S + i, ld};
+  // the model state in registers: every load of the instance is issued
+  // before the first dependent use (a global-memory accessor would interleave
+  // each load with the preceding stores: one memory round trip per entry)
+  double Sr[Tri<N>::size];
+#pragma unroll
+  for (int t = 0; t < Tri<N>::size; ++t) Sr[t] = st.S[(int64_t)t * ld + i];
   double u0[N];
   InstantOut io{u_out + i, ahat_out ? ahat_out + i : nullptr, nullptr, rank_out ? rank_out + i : nullptr, ld, true};
-  control_instant<N, M>(P, 0.0, cap, w, RegArr<N>{mu_f}, mu_p, S, RegArr<N>{Sfp}, RegArr<N>{A0r}, fbar, p,
-                        RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
+  control_instant<N, M>(P, 0.0, cap, w, RegArr<N>{mu_f}, mu_p, RegArr<Tri<N>::size>{Sr}, RegArr<N>{Sfp},
+                        RegArr<N>{A0r}, fbar, p, RegArr<N>{thr}, RegArr<N>{thr_max}, s_prev, act, u0, status, io);
+#pragma unroll
+  for (int t = 0; t < Tri<N>::size; ++t) st.S[(int64_t)t * ld + i] = Sr[t];
   st.w[i] = w;
   st.mu_p[i] = mu_p;
 #pragma unroll
@@ -1726,6 +1765,13 @@ __global__ void k_debug_gen(DevParams P, StatePtrs st, int64_t k, double *a_true
   c_true[i] = gen_c_true(P.seed, srv);
   noise[i] = gen_noise(gen_stream_key(P.seed, GEN_TAG_JIT, srv), k, P.noise_scale);
 }
+
+}  // namespace capgpu
+
+// the lane-parallel small-batch kernel (uses StatePtrs / TracePtrs and the device math above)
+#include "capgpu_lanes.cuh"
+
+namespace capgpu {
 
 // ------------------------------------------------------------------ launchers
 
@@ -1912,6 +1958,9 @@ int sim_occupancy(int block, int n_class) {
   return nb;
 }
 
+// instances up to which the lane-parallel kernel runs (env CAPGPU_LP_MAX_INST overrides)
+constexpr int64_t kLpMaxInst = 2048;
+
 template <int N, int M>
 struct LaunchNM {
   template <int S>
@@ -1943,6 +1992,19 @@ struct LaunchNM {
       return (int)cudaErrorInvalidConfiguration;
     }
     if (P.slo) return launch_sim<N, M, S, 32, true>(P, st, tr, k0, K, s);  // NEXT-1 (one block size)
+    // small batches: one lane per knob (k_simulate_lp, bitwise identical results)
+    if constexpr (S == 4) {
+      static int64_t lp_max = -1;
+      if (lp_max < 0) {
+        const char *e = getenv("CAPGPU_LP_MAX_INST");
+        lp_max = e ? atoll(e) : kLpMaxInst;
+      }
+      if (P.convex && !P.ref && P.n_inst <= lp_max) {
+        constexpr int G = N <= 4 ? 4 : (N <= 8 ? 8 : 16);
+        k_simulate_lp<N, M, S, G><<<grid_for(P.n_inst * G, 128), 128, 0, s>>>(P, st, tr, k0, K);
+        return (int)cudaGetLastError();
+      }
+    }
     if (occ128[nc] <= 0 || busiest(occ32[nc], 32) < busiest(occ128[nc], 128))
       return launch_sim<N, M, S, 32>(P, st, tr, k0, K, s);
     return launch_sim<N, M, S, 128>(P, st, tr, k0, K, s);
