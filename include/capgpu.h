@@ -271,6 +271,25 @@ int capgpu_tree_sum_host(const double *v, int64_t n, double *out);
 int capgpu_sim_state(capgpu_ctx *ctx, double *fbar_d, double *acc_d, double *thr_d, double *p_d,
                      void *stream);
 
+/* NEXT-3 explicit (multi-parametric) MPC ("an offline part and an
+ * online part ... solved incrementally as a piecewise linear function").
+ * Offline: from the context's current model state (the S1 solve: A-hat, as the
+ * next control_step would compute it before its push) and the weights of
+ * thr_d / thr_max_d [N][n] (S2), tabulate every server's applied control law
+ * u_0(beta) of Eq. 9's first block (weight c_0): the critical regions are
+ * nested in the tracking offset beta = p - P_s - A.f (knobs reach f_max in the
+ * stable ascending order of b_j = (f_max - f_min) / (c_0 tau_j)), each with an
+ * affine law.  The table (6N + 3 doubles per server) is owned by the context.
+ * Online: u_out [N][n] (device) = the law at beta of p_meas [n], f_applied
+ * [N][n], cap [n]; active_out [n] = block 0's 2-bit codes; status_out
+ * (nullable) = CAP_INFEASIBLE as control_step.  No model update, no weights
+ * (they are frozen in the table until the next build).  Convex literal Eq. 9
+ * only (no f_lo / ref_alpha / wmove: CAPGPU_E_UNSUPPORTED); CAPGPU_E_ORDER
+ * before identify/set_prior (build) or before a build (step). */
+int capgpu_explicit_build(capgpu_ctx *ctx, const double *thr_d, const double *thr_max_d, void *stream);
+int capgpu_explicit_step(capgpu_ctx *ctx, const double *p_meas_d, const double *f_applied_d, const double *cap_d,
+                         double *u_out_d, uint32_t *active_out_d, uint32_t *status_out_d, void *stream);
+
 /* Overwrite the plant state of the simulation (inverse of capgpu_sim_state;
  * device pointers, each nullable = keep).  Validated before anything is
  * written (synchronous on `stream`): every value finite and |acc_j| <=

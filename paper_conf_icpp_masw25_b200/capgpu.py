@@ -79,7 +79,7 @@ SYMBOLS = ["capgpu_version", "capgpu_status_string", "capgpu_last_error", "capgp
            "capgpu_sim_reset", "capgpu_sim_state", "capgpu_sim_caps", "capgpu_nccl_unique_id", "capgpu_shard_range",
            "capgpu_debug_gen", "capgpu_fp64_peak", "capgpu_simulate_group", "capgpu_tree_sum_host",
            "capgpu_debug_phase_counters", "capgpu_set_state", "capgpu_checkpoint_bytes", "capgpu_checkpoint_save",
-           "capgpu_checkpoint_load"]
+           "capgpu_checkpoint_load", "capgpu_explicit_build", "capgpu_explicit_step"]
 
 _lib = None
 
@@ -118,6 +118,8 @@ def lib():
     L.capgpu_sim_state.argtypes = [_VP, _VP, _VP, _VP, _VP, _VP]
     L.capgpu_sim_caps.argtypes = [_VP, _VP, _VP]
     L.capgpu_set_state.argtypes = [_VP, _VP, _VP, _VP, _VP, _VP]
+    L.capgpu_explicit_build.argtypes = [_VP, _VP, _VP, _VP]
+    L.capgpu_explicit_step.argtypes = [_VP, _VP, _VP, _VP, _VP, _VP, _VP, _VP]
     L.capgpu_checkpoint_bytes.argtypes = [_VP]
     L.capgpu_checkpoint_bytes.restype = C.c_int64
     L.capgpu_checkpoint_save.argtypes = [_VP, _VP, _VP]
@@ -383,6 +385,20 @@ class CapGPU:
         f, a, t, p = self._z(N, ni), self._z(N, ni), self._z(N, ni), self._z(ni)
         _check(self.L.capgpu_sim_state(self._ctx, _ptr(f), _ptr(a), _ptr(t), _ptr(p), _stream()), self._ctx)
         return dict(fbar=f, acc=a, thr=t, p=p)
+
+    def explicit_build(self, thr, thr_max):
+        """NEXT-3 explicit MPC, offline part: tabulate each server's piecewise-affine law."""
+        _check(self.L.capgpu_explicit_build(self._ctx, _ptr(thr), _ptr(thr_max), _stream()), self._ctx)
+
+    def explicit_step(self, p_meas, f_applied, cap):
+        """NEXT-3 explicit MPC, online part: u_0 = law(beta) by table lookup."""
+        n = self.n_srv
+        u = self._z(self.N, n)
+        act = self._z(n, dtype=torch.int32)
+        st = self._z(n, dtype=torch.int32)
+        _check(self.L.capgpu_explicit_step(self._ctx, _ptr(p_meas), _ptr(f_applied), _ptr(cap), _ptr(u), _ptr(act),
+                                           _ptr(st), _stream()), self._ctx)
+        return dict(u=u, active=act, status=st)
 
     def set_state(self, fbar=None, acc=None, thr=None, p=None):
         _check(self.L.capgpu_set_state(self._ctx, _ptr(fbar), _ptr(acc), _ptr(thr), _ptr(p), _stream()), self._ctx)

@@ -34,6 +34,8 @@ struct capgpu_ctx {
   int64_t k_global = 0;
   capgpu_workload wl{};
   Budget budget{};
+  double *explicit_tab = nullptr;  // NEXT-3 explicit MPC tables (allocated by the first capgpu_explicit_build)
+  bool explicit_ready = false;
   char err[512] = {0};
 };
 
@@ -413,6 +415,7 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
 int capgpu_destroy(capgpu_ctx *c) {
   if (!c) return CAPGPU_OK;
   budget_free(c->budget);
+  if (c->explicit_tab) cudaFree(c->explicit_tab);
   if (c->ws) cudaFree(c->ws);
   delete c;
   return CAPGPU_OK;
@@ -514,6 +517,47 @@ int capgpu_control_step(capgpu_ctx *c, const double *p_meas_d, const double *f_a
   int e = c->L.control_step(dp, c->st, p_meas_d, f_applied_d, thr_d, thr_max_d, cap_d, u_out_d, active_out_d,
                             rank_out_d, ahat_out_d, status_out_d, (cudaStream_t)stream);
   if (e) return cuda_fail(c, (cudaError_t)e, "control_step");
+  return CAPGPU_OK;
+}
+
+// NEXT-3 explicit (multi-parametric) MPC: offline part + online part
+int capgpu_explicit_build(capgpu_ctx *c, const double *thr_d, const double *thr_max_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  if (c->prm.caps_per_server != 1) return fail(c, CAPGPU_E_INVALID, "explicit MPC needs caps_per_server == 1");
+  NEED_DEV(c, thr_d);
+  NEED_DEV(c, thr_max_d);
+  if (!c->has_prior) return fail(c, CAPGPU_E_ORDER, "no prior A0: call capgpu_identify or capgpu_set_prior first");
+  if (!c->convex_static || c->prm.ref_alpha > 0.0 || c->prm.wmove > 0.0)
+    return fail(c, CAPGPU_E_UNSUPPORTED, "explicit MPC tabulates the convex literal Eq. 9 (no f_lo, reference "
+                                         "trajectory or move suppression)");
+  if (!c->explicit_tab) {
+    const size_t bytes = sizeof(double) * (size_t)c->L.explicit_fields * (size_t)c->n_srv;
+    cudaError_t e = cudaMalloc(&c->explicit_tab, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      c->explicit_tab = nullptr;
+      return fail(c, CAPGPU_E_NOMEM, "explicit table (%zu bytes): %s", bytes, cudaGetErrorString(e));
+    }
+  }
+  int e = c->L.explicit_build(c->dp, c->st, thr_d, thr_max_d, c->explicit_tab, (cudaStream_t)stream);
+  if (e) return cuda_fail(c, (cudaError_t)e, "explicit_build");
+  c->explicit_ready = true;
+  return CAPGPU_OK;
+}
+
+int capgpu_explicit_step(capgpu_ctx *c, const double *p_meas_d, const double *f_applied_d, const double *cap_d,
+                         double *u_out_d, uint32_t *active_out_d, uint32_t *status_out_d, void *stream) {
+  if (!c) return fail(nullptr, CAPGPU_E_INVALID, "ctx is NULL");
+  NEED_DEV(c, p_meas_d);
+  NEED_DEV(c, f_applied_d);
+  NEED_DEV(c, cap_d);
+  NEED_DEV(c, u_out_d);
+  NEED_DEV(c, active_out_d);
+  OPT_DEV(c, status_out_d);
+  if (!c->explicit_ready) return fail(c, CAPGPU_E_ORDER, "no explicit table: call capgpu_explicit_build first");
+  int e = c->L.explicit_step(c->dp, c->explicit_tab, p_meas_d, f_applied_d, cap_d, u_out_d, active_out_d,
+                             status_out_d, (cudaStream_t)stream);
+  if (e) return cuda_fail(c, (cudaError_t)e, "explicit_step");
   return CAPGPU_OK;
 }
 

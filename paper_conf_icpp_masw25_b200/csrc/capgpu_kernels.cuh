@@ -1715,6 +1715,160 @@ __global__ void __launch_bounds__(128) k_control_step(DevParams P, StatePtrs st,
   if (status_out) status_out[i] = status;
 }
 
+// ------------------------------------------------------------------ explicit (multi-parametric) MPC (NEXT-3)
+//
+// "the MPC control problem [can be divided] into an offline part and an
+// online part, [solving] the online part incrementally as a piecewise linear
+// function".  For a fixed model A and weights R, the applied block of Eq. 9
+// (weight c = c_0) is a strictly convex box QP whose only varying parameter is
+// the scalar tracking offset beta = p(k) - P_s(k) - A.f(k): its solution is
+// piecewise affine in beta.  With l = m (no SLO bound, the convex case) the
+// critical regions are nested: knob j goes to its upper bound once -c s tau_j
+// > h_j - m_j, i.e. s < -b_j, b_j = (h_j - m_j) / (c tau_j), so region r
+// (r = 0..N) holds the r knobs with the smallest b (stable order) at h and
+// s_r(base) = (base + n_r) / D_r, base = beta + A.l, n_r = sum_{U_r} A_j (h_j - m_j),
+// D_r = 1 + c sum_{j not in U_r} tau_j A_j.
+// Offline (k_explicit_build): A from the model state (the S1 solve), tau from
+// the weights of thr/thr_max (S2), the stable rank of each b_j and, per
+// region, n_r, 1/D_r and the lower end T_r = -b_(r) D_r - n_r of the region in
+// base (-inf for the last region).  Online (k_explicit_step): base, the region
+// r* = #{r < N : base < T_r} (branch-free), s = (base + n_r*) / D_r*, u_j =
+// h_j if rank_j < r* else m_j - c tau_j s; base >= 0: every knob at l.
+// Table per server (SoA [field][n_srv]): A[N] | tau[N] | rank[N] (as double) |
+// n[N+1] | invD[N+1] | T[N+1].
+template <int N>
+struct ExplicitTable {
+  static constexpr int oA = 0, oTau = N, oRank = 2 * N, oN = 3 * N, oInvD = 4 * N + 1, oT = 5 * N + 2,
+                       fields = 6 * N + 3;
+};
+
+template <int N>
+__global__ void __launch_bounds__(128) k_explicit_build(DevParams P, StatePtrs st, const double *thr_in,
+                                                        const double *thr_max_in, double *tab) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= P.n_srv) return;
+  const int64_t ld = P.n_srv;
+  using ET = ExplicitTable<N>;
+  // S1 solve from the stored model state (model_solve, unscaled as control_step)
+  double Sr[Tri<N>::size], Sfp[N], A0r[N], ahat[N];
+#pragma unroll
+  for (int t = 0; t < Tri<N>::size; ++t) Sr[t] = st.S[(int64_t)t * ld + i];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    Sfp[j] = st.Sfp[j * ld + i];
+    A0r[j] = st.A0[j * ld + i];
+  }
+  model_solve<N>(P.rho, P.a_lo, P.a_hi, RegArr<Tri<N>::size>{Sr}, RegArr<N>{Sfp}, RegArr<N>{A0r}, ahat);
+  // S2 weights (IEEE, as the reported theta) -> tau_j = A_j theta_j / r0_j
+  const double c = P.ct[0];
+  double tau[N], b[N], ta[N], ad[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    const double th = pclamp(__ddiv_rn(thr_in[j * ld + i], thr_max_in[j * ld + i]), P.theta_min, 1.0);
+    tau[j] = ahat[j] * th * P.k[j].inv_r0;
+    ta[j] = tau[j] * ahat[j];
+    ad[j] = ahat[j] * P.k[j].span;
+    b[j] = tau[j] > 0.0 ? P.k[j].span / (c * tau[j]) : INFINITY;  // s < -b_j: knob j upper
+  }
+  // stable ascending ranks of b (ties -> lower knob index)
+  int rk[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    int r = 0;
+#pragma unroll
+    for (int q = 0; q < N; ++q) r += (b[q] < b[j]) || (q < j && b[q] == b[j]);
+    rk[j] = r;
+  }
+  double TA = 0.0;
+#pragma unroll
+  for (int j = 0; j < N; ++j) TA += ta[j];
+#pragma unroll
+  for (int r = 0; r <= N; ++r) {
+    double nr = 0.0, tu = 0.0, br = INFINITY;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      if (rk[j] < r) {
+        nr += ad[j];
+        tu += ta[j];
+      }
+      if (rk[j] == r) br = b[j];
+    }
+    const double D = fma(c, TA - tu, 1.0);
+    tab[(int64_t)(ET::oN + r) * ld + i] = nr;
+    tab[(int64_t)(ET::oInvD + r) * ld + i] = 1.0 / D;
+    tab[(int64_t)(ET::oT + r) * ld + i] = r < N && br < INFINITY ? fma(-br, D, -nr) : -INFINITY;
+  }
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    tab[(int64_t)(ET::oA + j) * ld + i] = ahat[j];
+    tab[(int64_t)(ET::oTau + j) * ld + i] = tau[j];
+    tab[(int64_t)(ET::oRank + j) * ld + i] = (double)rk[j];
+  }
+}
+
+template <int N>
+__global__ void __launch_bounds__(128) k_explicit_step(DevParams P, const double *tab, const double *p_meas,
+                                                       const double *f_app, const double *cap_in, double *u_out,
+                                                       uint32_t *act_out, uint32_t *status_out) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= P.n_srv) return;
+  const int64_t ld = P.n_srv;
+  using ET = ExplicitTable<N>;
+  double a[N], tau[N], f[N], T[N + 1], nr[N + 1], iD[N + 1];
+  int rk[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    a[j] = tab[(int64_t)(ET::oA + j) * ld + i];
+    tau[j] = tab[(int64_t)(ET::oTau + j) * ld + i];
+    rk[j] = (int)tab[(int64_t)(ET::oRank + j) * ld + i];
+    f[j] = f_app[j * ld + i];
+  }
+#pragma unroll
+  for (int r = 0; r <= N; ++r) {
+    T[r] = tab[(int64_t)(ET::oT + r) * ld + i];
+    nr[r] = tab[(int64_t)(ET::oN + r) * ld + i];
+    iD[r] = tab[(int64_t)(ET::oInvD + r) * ld + i];
+  }
+  const double p = p_meas[i], cap = cap_in[i];
+  double beta = p - cap, smin = 0.0, smax = 0.0;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    beta = fma(-a[j], f[j], beta);
+    smin = fma(a[j], P.k[j].lo, smin);
+    smax = fma(a[j], P.k[j].hi, smax);
+  }
+  const uint32_t status = (beta + smin > 0.0 || beta + smax < 0.0) ? (uint32_t)CAPGPU_ST_CAP_INFEASIBLE : 0u;
+  const double base = beta + smin;
+  uint32_t code = 0u;
+  if (!(base < 0.0)) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      code |= (base > 0.0 && tau[j] > 0.0 ? 1u : 0u) << (2 * j);
+      u_out[j * ld + i] = P.k[j].lo;
+    }
+  } else {
+    int r = 0;  // the region: #{r < N : base < T_r} (T decreasing in r)
+#pragma unroll
+    for (int q = 0; q < N; ++q) r += base < T[q];
+    double n = nr[0], id = iD[0];
+#pragma unroll
+    for (int q = 1; q <= N; ++q) {
+      n = r == q ? nr[q] : n;
+      id = r == q ? iD[q] : id;
+    }
+    const double s = (base + n) * id;
+    const double mcs = -P.ct[0] * s;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const bool up = rk[j] < r;
+      code |= (up ? 2u : 0u) << (2 * j);
+      u_out[j * ld + i] = up ? P.k[j].hi : fma(mcs, tau[j], P.k[j].m);
+    }
+  }
+  act_out[i] = code;
+  if (status_out) status_out[i] = status;
+}
+
 template <int N>
 __global__ void k_assign_weights(DevParams P, const double *thr_in, const double *thr_max_in, double *theta_out,
                                  double *R_out, int8_t *rank_out, int64_t n) {
@@ -1792,6 +1946,10 @@ struct Launchers {
                 cudaStream_t);
   int (*budget_init)(const DevParams &, const StatePtrs &, const BudgetDev &, double *, cudaStream_t);
   int (*baseline)(const DevParams &, const StatePtrs &, const TracePtrs &, int64_t, int, cudaStream_t);
+  int (*explicit_build)(const DevParams &, const StatePtrs &, const double *, const double *, double *, cudaStream_t);
+  int (*explicit_step)(const DevParams &, const double *, const double *, const double *, const double *, double *,
+                       uint32_t *, uint32_t *, cudaStream_t);
+  int explicit_fields;
 };
 
 inline int grid_for(int64_t n, int block) { return (int)((n + block - 1) / block); }
@@ -1831,6 +1989,16 @@ struct LaunchN {
                       cudaStream_t s) {
     if (P.S == 4) return P.slo ? baseline_s<4, true>(P, st, tr, k0, K, s) : baseline_s<4, false>(P, st, tr, k0, K, s);
     return P.slo ? baseline_s<0, true>(P, st, tr, k0, K, s) : baseline_s<0, false>(P, st, tr, k0, K, s);
+  }
+  static int explicit_build(const DevParams &P, const StatePtrs &st, const double *thr, const double *tm,
+                            double *tab, cudaStream_t s) {
+    k_explicit_build<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, st, thr, tm, tab);
+    return (int)cudaGetLastError();
+  }
+  static int explicit_step(const DevParams &P, const double *tab, const double *p, const double *f, const double *cap,
+                           double *u, uint32_t *act, uint32_t *status, cudaStream_t s) {
+    k_explicit_step<N><<<grid_for(P.n_srv, 128), 128, 0, s>>>(P, tab, p, f, cap, u, act, status);
+    return (int)cudaGetLastError();
   }
   static int budget_init(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, double *part_c,
                          cudaStream_t s) {
@@ -2045,6 +2213,9 @@ Launchers make_launchers(int M) {
   L.debug_gen = &LaunchN<N>::debug_gen;
   L.budget_init = &LaunchN<N>::budget_init;
   L.baseline = &LaunchN<N>::baseline;
+  L.explicit_build = &LaunchN<N>::explicit_build;
+  L.explicit_step = &LaunchN<N>::explicit_step;
+  L.explicit_fields = ExplicitTable<N>::fields;
 #define CAPGPU_SET_M(MM)                                 \
   case MM:                                               \
     L.simulate = &LaunchNM<N, MM>::simulate;             \

@@ -1,10 +1,13 @@
 #!/bin/bash
-# GPU-box round check: full GPU suite, smoke, bench lines (cfg 3 default, cfg 5, cfg 4),
-# ncu launch list of the default bench command.
+# GPU-box round check: full GPU suite, smoke, bench lines (cfg 3 default, cfg 5, cfg 4, cfg 2, slo,
+# control_step), ncu launch list of the default bench command.
 mkdir -p gpurun_out
-timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -2 gpurun_out/smoke.log
-timeout 600 python bench.py > gpurun_out/bench_cfg3.json 2> gpurun_out/bench_cfg3.err; echo "bench rc=$?"; cat gpurun_out/bench_cfg3.json
-timeout 600 python bench.py --config 5 --no-cpu-baseline > gpurun_out/bench_cfg5.json 2> gpurun_out/bench_cfg5.err; cat gpurun_out/bench_cfg5.json
-timeout 600 python bench.py --config 4 --no-cpu-baseline > gpurun_out/bench_cfg4.json 2> gpurun_out/bench_cfg4.err; cat gpurun_out/bench_cfg4.json
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_cfg3.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_launch_bench.log 2>&1; echo "ncu rc=$?"
+TAG=${TAG:-r2}
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu_$TAG.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu_$TAG.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_$TAG.log 2>&1; echo "smoke rc=$?"; tail -2 gpurun_out/smoke_$TAG.log
+timeout 600 python bench.py > gpurun_out/bench_cfg3_$TAG.json 2> gpurun_out/bench_cfg3_$TAG.err; echo "bench rc=$?"; cat gpurun_out/bench_cfg3_$TAG.json
+for c in 5 4 2 slo; do
+  timeout 600 python bench.py --config $c --no-cpu-baseline > gpurun_out/bench_cfg${c}_$TAG.json 2> gpurun_out/bench_cfg${c}_$TAG.err; cat gpurun_out/bench_cfg${c}_$TAG.json
+done
+timeout 300 python bench.py --config 3 --call control_step --no-cpu-baseline --steps 50 > gpurun_out/bench_cs_$TAG.json 2> gpurun_out/bench_cs_$TAG.err; cat gpurun_out/bench_cs_$TAG.json
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_cfg3_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_launch_bench_$TAG.log 2>&1; echo "ncu rc=$?"
