@@ -3,7 +3,7 @@ libcapgpu_timing.so, -DCAPGPU_PHASE_TIMING).  Prints the share of each phase
 of the period loop, averaged over instances.
 
     python -m paper_conf_icpp_masw25_b200.build --variant=timing
-    CAPGPU_LIB_VARIANT=timing python tools/phase_timing.py [cfg] [periods]
+    CAPGPU_LIB_VARIANT=timing python tools/phase_timing.py [cfg] [periods] [n_servers]
 """
 import os
 import sys
@@ -23,8 +23,9 @@ NAMES = {1: "S1 Welford push", 2: "S1 LDL^T solve + clamp", 3: "S2 weights (+tra
 
 cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 3
 periods = int(sys.argv[2]) if len(sys.argv) > 2 else 200
+n_srv = int(sys.argv[3]) if len(sys.argv) > 3 else None  # e.g. 4736 = one warp per SM (latency chain alone)
 d = configs.get(cfg)
-g = G.CapGPU.from_config(d)
+g = G.CapGPU.from_config(d, n_servers=n_srv)
 wl = G.workload_from(d)
 g.simulate(periods, wl)  # init + warm
 cnt = torch.zeros(8, g.n_inst, dtype=torch.int64, device="cuda")
