@@ -12,7 +12,7 @@ S1-S4 per step.  Default workload: BASELINE.json configs[2]
 demand and throughput-driven weights) - see DESIGN.md §8 for why cfg 3.
 
 Timing: W untimed warm-up steps, then K timed steps, each bracketed by CUDA
-events on the launching stream; L2 is flushed (256 MiB write) between timed
+events on the launching stream; L2 is flushed (256 MiB write + read) between timed
 steps outside the events; barrier + synchronize on both sides; max over ranks.
 Multi-GPU (torchrun): one process per GPU.  Strong scaling:
 the SAME global problem is split into contiguous 1024-server shards
@@ -127,6 +127,29 @@ class ClockSampler(threading.Thread):
                 "samples": len(win)}
 
 
+FLUSH_MODE = os.environ.get("CAPGPU_BENCH_FLUSH", "write+read")
+
+
+L2_DESC = {"write+read": "flushed between timed steps (256 MiB write + read of it outside the events: L2 cold and clean)",
+           "write": "flushed between timed steps (256 MiB write outside the events)",
+           "none": "NOT flushed (A/B only)"}.get(FLUSH_MODE, FLUSH_MODE)
+
+
+def l2_flush(buf):
+    """L2 flush between timed steps (outside the events): a 256 MiB write
+    (evicts every line of the 126 MB L2), then a read of the same buffer so the
+    L2 is left cold AND clean: without the read, the next timed step pays the
+    write-back of up to 126 MB of the flush buffer's dirty lines (measured on
+    capgpu_control_step at the cfg 3 shape: 31.9 us per call after the write
+    alone, 29.5 after write + read, 25.6 with no flush).
+    CAPGPU_BENCH_FLUSH=write restores the write-only flush, =none skips it (A/B only)."""
+    if FLUSH_MODE == "none":
+        return
+    buf.zero_()
+    if FLUSH_MODE == "write+read":
+        buf.sum()
+
+
 # ---------------------------------------------------------------- oracle (CPU baseline / reference arm)
 
 def _oracle_worker(args):
@@ -233,7 +256,7 @@ def bench_control_step(args, d, g, world, rank, local, dev, n_global):
     barrier()
     t0 = time.monotonic()
     for i in range(args.steps):
-        flush.zero_()
+        l2_flush(flush)
         evs[i][0].record(stream)
         g.control_step(devb["p"], devb["f"], devb["thr"], devb["thr_max"], devb["cap"], out=obuf)
         evs[i][1].record(stream)
@@ -251,7 +274,7 @@ def bench_control_step(args, d, g, world, rank, local, dev, n_global):
     u_host = torch.empty(N, n, dtype=torch.float64, pin_memory=True)
     e2e = []
     for _ in range(max(3, args.steps // 2)):
-        flush.zero_()
+        l2_flush(flush)
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         for k in devb:
@@ -277,7 +300,7 @@ def bench_control_step(args, d, g, world, rank, local, dev, n_global):
                 "config": {"workload": f"capgpu_control_step at the cfg{d['cfg']} shape: {n_global:,} servers, "
                                        f"N={N}, P/M={d['P']}/{M} (S1-S3 per call, state in HBM)",
                            "instances_per_gpu": n, "mode": "per-period C-ABI call k_control_step (1 launch per step)",
-                           "l2": "flushed between timed steps (256 MiB write outside the events)",
+                           "l2": L2_DESC,
                            "parallelism": f"dp{world}"},
                 "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                              "frac": achieved / peak, "traffic": None, "bytes_per_step": bps,
@@ -421,7 +444,7 @@ def main():
     barrier()
     t0 = time.monotonic()
     for i in range(args.steps):
-        flush.zero_()  # L2 flush outside the timed events
+        l2_flush(flush)  # L2 flush outside the timed events
         evs[i][0].record(stream)
         g.simulate(periods, wl, out=bufs)
         evs[i][1].record(stream)
@@ -448,7 +471,7 @@ def main():
                  for k, dt in (("sum_p", torch.float64), ("max_p", torch.float64), ("n_viol", torch.int32))}
     e2e_evs = []
     for i in range(max(3, args.steps // 2)):
-        flush.zero_()
+        l2_flush(flush)
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         if not hier:
@@ -531,7 +554,7 @@ def main():
                            "mode": mode,
                            "global_instances": (n_global * caps if not hier else n_global),
                            "per_period_us": 1e6 * t_max / args.steps / periods,
-                           "l2": "flushed between timed steps (256 MiB write outside the events)",
+                           "l2": L2_DESC,
                            "parallelism": par},
                 "roofline": roof,
                 "e2e": {"value": e2e_value, "unit": "server-control-steps/s",

@@ -357,8 +357,11 @@ int capgpu_create(capgpu_ctx **out, int64_t n_servers, int32_t n_gpus, capgpu_ho
   s.thr = take(N * ni);
   s.p = take(ni);
   s.w = take(ni);
-  s.mu_f = take(N * ni);
   s.mu_p = take(ni);
+  // mu_f | Sigma | Sigma_fp are consecutive rows (ld n_inst) and a_true ..
+  // A0 below are consecutive rows (ld n_srv): k_period stages each block
+  // with one 2D TMA box per 32 servers
+  s.mu_f = take(N * ni);
   s.S = take(c->T * ni);
   s.Sfp = take(N * ni);
   s.cap_base = take(ni);

@@ -466,8 +466,11 @@ __device__ __forceinline__ double solve_block(const KnobConst *kc, const KnobCon
 #pragma unroll
   for (int j = 0; j < N; ++j) cta[j] = ctau[j] * a[j];
   double s = s_warm;
+#ifndef CAPGPU_NEWTON_TRIES  // 3 / 4 / 6 tries measured 5 / 9 / 16 % slower on the SLO bench (lanes that
+#define CAPGPU_NEWTON_TRIES 2  // leave Newton's first two pieces oscillate; tools/ab_slo.sh)
+#endif
 #pragma unroll 1
-  for (int it = 0; it < 2; ++it) {
+  for (int it = 0; it < CAPGPU_NEWTON_TRIES; ++it) {
     double phi, slope;
     const uint32_t c0 = block_eval<N>(kc, a, ctau, cta, beta, s, phi, slope);
     if (phi == 0.0) return s;

@@ -15,6 +15,8 @@
 #include <algorithm>
 #include <cmath>
 
+#include <cuda.h>  // CUtensorMap (the encoder is fetched from the driver at run time: no -lcuda)
+
 #include "capgpu_device.cuh"
 
 namespace capgpu {
@@ -657,6 +659,14 @@ struct SimOccupancy {
 #else
   static constexpr int warps = N <= 4 ? 16 : (N <= 6 ? 12 : 8);
 #endif
+  // The SLO-schedule instantiation (general block solve, out-of-line exact
+  // fallback) spills at 128 registers: 12 warps (168 registers) measured
+  // 10.42 vs 8.71 G steps/s at 16 and 9.29 at 8 (N = 4, tools/ab_slo.sh).
+#ifdef CAPGPU_SLO_WARPS
+  static constexpr int slo_warps = CAPGPU_SLO_WARPS < warps ? CAPGPU_SLO_WARPS : warps;
+#else
+  static constexpr int slo_warps = warps < 12 ? warps : 12;
+#endif
 };
 
 // SLO: the NEXT-1 SLO-schedule instantiation (phase tracking, per-phase bounds,
@@ -956,7 +966,7 @@ __device__ __forceinline__ void sim_run(const DevParams &P, const StatePtrs &st,
 }
 
 template <int N, int M, int S, int BLOCK, bool SLO = false, bool MOVE = false, bool CH = false>
-__global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : SimOccupancy<N>::warps) * 32 / BLOCK)
+__global__ void __launch_bounds__(BLOCK, (MOVE ? 8 : (SLO ? SimOccupancy<N>::slo_warps : SimOccupancy<N>::warps)) * 32 / BLOCK)
     k_simulate(DevParams P, StatePtrs st, TracePtrs tr, int64_t k0, int K, SimSched sc) {
   extern __shared__ __align__(16) double smem[];
   double *my = smem + threadIdx.x * SlabLayout<N>::F;
@@ -1290,15 +1300,24 @@ struct TileAcc {
 template <int N>
 struct PeriodTile {
   static constexpr int T = Tri<N>::size;
-  // Sigma | mu_f | Sfp | A0 | thr_max | base | amp | a_true | C_true; the
-  // read-only constants are staged only when the tile fits the 227 KB of
-  // shared memory, else they are read from global memory where used.
+  // Two blocks of workspace rows, in workspace order (one 2D TMA box each):
+  // the model mu_f | Sigma | Sfp (ld n_inst) and the read-only constants
+  // a_true | C_true | thr_max | base | amp | A0 (ld n_srv).  The constants are
+  // staged only when the tile fits the 227 KB of shared memory, else they are
+  // read from global memory where used.
   // (kPeriodWarps > 8, an experiment build: the tiles of all resident warps must fit)
   static constexpr bool ro =
       (T + 7 * N + 1) * kPeriodCta * 8 * (kPeriodWarps > 8 ? kPeriodWarps * 32 / kPeriodCta : 1) <= 227 * 1024;
-  static constexpr int oS = 0, oMU = T, oSFP = T + N, oA0 = T + 2 * N, oTM = T + 3 * N, oBA = T + 4 * N,
-                       oAM = T + 5 * N, oAT = T + 6 * N, oCT = T + 7 * N, F = ro ? T + 7 * N + 1 : T + 2 * N;
+  static constexpr int oMU = 0, oS = N, oSFP = N + T, MODEL = 2 * N + T, oAT = MODEL, oCT = MODEL + N,
+                       oTM = MODEL + N + 1, oBA = MODEL + 2 * N + 1, oAM = MODEL + 3 * N + 1, oA0 = MODEL + 4 * N + 1,
+                       RO = 5 * N + 1, F = ro ? MODEL + RO : MODEL;
   static constexpr int bytes_per_cta = F * kPeriodCta * 8;
+};
+
+// tensor maps of the two staged row blocks (k_period; ok = false: per-thread cp.async)
+struct PeriodMaps {
+  CUtensorMap model, ro;
+  int ok;
 };
 
 template <bool RO>
@@ -1349,6 +1368,15 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned by
                : "memory");
 }
 
+// 2D TMA box load (global -> shared, mbarrier completion); x = server, y = row
+__device__ __forceinline__ void tma_box(void *dst, const CUtensorMap *map, int x, int y, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
+      : "memory");
+}
+
 // cp.async of the server's model state and read-only constants into its tile
 // column (tile = warp tile base + lane)
 template <int N>
@@ -1371,37 +1399,25 @@ __device__ __forceinline__ void period_stage(const StatePtrs &st, int64_t i, int
   if constexpr (PT::ro) cp_async8(tile + PT::oCT * 32, st.c_true + i);
 }
 
-// The same staging for a whole warp of 32 consecutive servers (i0 = first,
-// 16-byte aligned rows): lane 0 arms the warp's mbarrier with the tile's
-// byte count and issues one 256-byte TMA bulk copy per field row (the SoA row
-// of 32 servers is contiguous).  The copies bypass L1 (the per-thread 8-byte
+// The same staging for a whole warp of 32 consecutive servers (i0 = first):
+// lane 0 arms the warp's mbarrier with the tile's byte count and issues one
+// 2D TMA box per row block (32 servers x the model rows, 32 servers x the
+// read-only rows): two instructions instead of one bulk copy per 256-byte
+// field row (which cost ~10 issue slots each behind lane 0, ~900 warp
+// instructions per period).  The boxes bypass L1 (the per-thread 8-byte
 // cp.async of the fallback allocate L1 lines, of which ~28 KB are left beside
 // the 8 tiles: that capped the bytes in flight, VERDICT r1 / ncu
-// long_scoreboard 3.5 per issue).
+// long_scoreboard 3.5 per issue).  Servers past n_srv in a ragged last warp
+// are zero-filled by the TMA unit (and never stored).
 template <int N>
-__device__ __forceinline__ void period_stage_tma(const StatePtrs &st, int64_t i0, int64_t ld, double *wtile,
-                                                 uint64_t *bar) {
+__device__ __forceinline__ void period_stage_tma(const PeriodMaps &pm, int64_t i0, double *wtile, uint64_t *bar) {
   using PT = PeriodTile<N>;
   if ((threadIdx.x & 31) == 0) {
     mbar_init(bar, 1);
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     mbar_arrive_expect_tx(bar, (unsigned)(PT::F * 32 * 8));
-    auto row = [&](int t, const double *g) { bulk_g2s(wtile + t * 32, g + i0, 256u, bar); };
-#pragma unroll 1
-    for (int t = 0; t < PT::T; ++t) row(PT::oS + t, st.S + t * ld);
-#pragma unroll 1
-    for (int j = 0; j < N; ++j) {
-      row(PT::oMU + j, st.mu_f + j * ld);
-      row(PT::oSFP + j, st.Sfp + j * ld);
-      if constexpr (PT::ro) {
-        row(PT::oA0 + j, st.A0 + j * ld);
-        row(PT::oTM + j, st.thr_max + j * ld);
-        row(PT::oBA + j, st.base + j * ld);
-        row(PT::oAM + j, st.amp + j * ld);
-        row(PT::oAT + j, st.a_true + j * ld);
-      }
-    }
-    if constexpr (PT::ro) row(PT::oCT, st.c_true);
+    tma_box(wtile, &pm.model, (int)i0, 0, bar);
+    if constexpr (PT::ro) tma_box(wtile + PT::oAT * 32, &pm.ro, (int)i0, 0, bar);
   }
   __syncwarp();
 }
@@ -1573,7 +1589,7 @@ __device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs 
 // budget caps, S1-S3, the w_i / p partial sums, S4.  State in HBM.
 template <int N, int M, int SS>
 __global__ void __launch_bounds__(kPeriodCta, kPeriodWarps * 32 / kPeriodCta) k_period(DevParams P, StatePtrs st, BudgetDev bd, TracePtrs tr, int64_t k,
-                                                int kk, int K) {
+                                                int kk, int K, const __grid_constant__ PeriodMaps pm) {
   if (bd.kdev) {  // graph replay: the period comes from device memory
     kk = (int)bd.kdev[1];
     k = bd.kdev[0] + kk;
@@ -1581,19 +1597,19 @@ __global__ void __launch_bounds__(kPeriodCta, kPeriodWarps * 32 / kPeriodCta) k_
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = i < P.n_srv;
   using PT = PeriodTile<N>;
-  extern __shared__ __align__(16) double ptile[];
+  extern __shared__ __align__(128) double ptile[];  // TMA tensor boxes land on 128-byte aligned rows
   double *tile = ptile + (threadIdx.x >> 5) * (PT::F * 32) + (threadIdx.x & 31);
   // Every load of the period is issued in one batch before anything waits:
   // the model state and read-only constants into this warp's tile
   // (asynchronous, no registers held), the rest into registers (one memory
   // round trip per server and period).
-  // full warps of 16-byte aligned rows: TMA bulk copies (one per field row);
-  // otherwise (ragged tail, odd server count) the per-thread cp.async
+  // TMA boxes when the host could encode the tensor maps (16-byte aligned
+  // rows: even server count); otherwise the per-thread cp.async
   __shared__ __align__(8) uint64_t wbar[kPeriodCta / 32];
   const int64_t i0 = i - (threadIdx.x & 31);
-  const bool bulk = (P.n_srv & 1) == 0 && i0 + 32 <= P.n_srv;
+  const bool bulk = pm.ok != 0;
   if (bulk)
-    period_stage_tma<N>(st, i0, P.n_srv, tile - (threadIdx.x & 31), &wbar[threadIdx.x >> 5]);
+    period_stage_tma<N>(pm, i0, tile - (threadIdx.x & 31), &wbar[threadIdx.x >> 5]);
   else if (valid)
     period_stage<N>(st, i, P.n_srv, tile);
   double tbar, p;
@@ -1954,6 +1970,36 @@ struct Launchers {
 
 inline int grid_for(int64_t n, int block) { return (int)((n + block - 1) / block); }
 
+// Host: 2D tensor map of `rows` SoA rows of `n` elements (leading dimension
+// `ld` elements, element size 8 or 4 bytes) starting at `base`, box = 32
+// elements x all rows (one TMA instruction per 32-column group).  Returns
+// false when TMA cannot describe it (misaligned base, stride not a multiple
+// of 16 bytes, > 256 rows, no driver entry point); the caller then uses its
+// non-TMA path.
+inline bool tma_map_2d(CUtensorMap *m, const void *base, uint64_t n, uint32_t rows, uint64_t ld, int esize = 8) {
+  using Enc = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                           const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                           CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static Enc enc = nullptr;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void *fn = nullptr;
+    cudaDriverEntryPointQueryResult q{};
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      enc = reinterpret_cast<Enc>(fn);
+    cudaGetLastError();
+  }
+  if (!enc || !base || ((uintptr_t)base & 15u) || rows == 0 || rows > 256 || (ld * esize) % 16 || n == 0) return false;
+  const cuuint64_t dims[2] = {n, rows}, strides[1] = {ld * (uint64_t)esize};
+  const cuuint32_t box[2] = {32, rows}, es[2] = {1, 1};
+  return enc(m, esize == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_UINT32, 2,
+             const_cast<void *>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 template <int N>
 struct LaunchN {
   static int init_servers(const DevParams &P, const StatePtrs &st, cudaStream_t s) {
@@ -2191,13 +2237,20 @@ struct LaunchNM {
   }
   static int period(const DevParams &P, const StatePtrs &st, const BudgetDev &bd, const TracePtrs &tr, int64_t k,
                     int kk, int K, cudaStream_t s) {
-    const int smem = PeriodTile<N>::bytes_per_cta;
+    using PT = PeriodTile<N>;
+    const int smem = PT::bytes_per_cta;
+    // the staged row blocks as 2D tensor maps (encoded on the host per launch;
+    // a CUDA graph captures them by value with the other parameters)
+    PeriodMaps pm{};
+    pm.ok = P.n_inst == P.n_srv && P.n_srv <= 0x7fffffffLL && !getenv("CAPGPU_PERIOD_NO_TMA") &&
+            tma_map_2d(&pm.model, st.mu_f, (uint64_t)P.n_srv, PT::MODEL, (uint64_t)P.n_inst) &&
+            (!PT::ro || tma_map_2d(&pm.ro, st.a_true, (uint64_t)P.n_srv, PT::RO, (uint64_t)P.n_srv));
     if (P.S == 4) {
       cudaFuncSetAttribute(k_period<N, M, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-      k_period<N, M, 4><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, smem, s>>>(P, st, bd, tr, k, kk, K);
+      k_period<N, M, 4><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, smem, s>>>(P, st, bd, tr, k, kk, K, pm);
     } else {
       cudaFuncSetAttribute(k_period<N, M, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-      k_period<N, M, 0><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, smem, s>>>(P, st, bd, tr, k, kk, K);
+      k_period<N, M, 0><<<grid_for(P.n_srv, kPeriodCta), kPeriodCta, smem, s>>>(P, st, bd, tr, k, kk, K, pm);
     }
     return (int)cudaGetLastError();
   }

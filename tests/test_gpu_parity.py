@@ -117,15 +117,17 @@ def test_assign_weights_bit_exact(G, oracle_mod):
 
 # ------------------------------------------------------------------ S1-S3 control step
 
-@pytest.mark.parametrize("n_gpus,P,M", [(1, 4, 2), (2, 4, 2), (4, 8, 2), (8, 8, 3), (3, 8, 1), (15, 8, 4)])
-def test_control_step_sequence(G, oracle_mod, n_gpus, P, M):
+@pytest.mark.parametrize("n_gpus,P,M,n", [(1, 4, 2, 133), (2, 4, 2, 133), (4, 8, 2, 133), (8, 8, 3, 133),
+                                           (3, 8, 1, 133), (15, 8, 4, 133),
+                                           # several full 128-server CTAs + a ragged tail
+                                           (8, 8, 3, 420), (3, 8, 2, 256)])
+def test_control_step_sequence(G, oracle_mod, n_gpus, P, M, n):
     """Several consecutive control_step calls on random measurements: model
     state, warm starts and all M blocks against the oracle's S1 (recursive),
     S2 and stacked S3."""
     d = desc_for(n_gpus, P=P, M=M)
     o = oracle_mod.Oracle(d)
     N = o.n
-    n = 133
     rng = np.random.default_rng(43 + N)
     g = G.CapGPU.from_config(d, n_servers=n)
     A0 = np.abs(np.where(np.arange(N)[:, None] == 0, 0.05, 0.2) * (1 + 0.2 * rng.standard_normal((N, n)))) + 1e-3
