@@ -160,6 +160,23 @@ __device__ __forceinline__ double rcp_nr1(double x) {
   return fma(y, fma(-x, y, 1.0), y);
 }
 
+// Position r = k mod cap_period in the cap step schedule of gen_cap_at,
+// advanced by one per period instead of a 64-bit modulo (a software division)
+// every period; the caps are bitwise those of gen_cap_at.  Used by the
+// latency-bound lane-parallel kernel (cfg 2: 1.45 -> 1.35 us per period with
+// the draws hoisted, capgpu_lanes.cuh); in k_simulate the extra live register
+// cost more than the modulo saved (cfgs 3/5 -1.2 / -1.5 %, no cap schedule).
+struct CapSched {
+  int64_t r;
+  __device__ __forceinline__ CapSched(const DevParams &P, int64_t k) : r(P.cap_period > 0 ? k % P.cap_period : 0) {}
+  __device__ __forceinline__ double cap(const DevParams &P, double base) const {
+    return (P.cap_period > 0 && r >= P.cap_lo && r < P.cap_hi) ? GEN_MUL(base, P.cap_mult) : base;
+  }
+  __device__ __forceinline__ void next(const DevParams &P) {
+    if (P.cap_period > 0 && ++r == P.cap_period) r = 0;
+  }
+};
+
 __device__ __forceinline__ long long dbits(double x) { return __double_as_longlong(x); }
 __device__ __forceinline__ double bitsd(long long b) { return __longlong_as_double(b); }
 

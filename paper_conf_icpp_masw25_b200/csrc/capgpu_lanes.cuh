@@ -140,10 +140,34 @@ __global__ void __launch_bounds__(128) k_simulate_lp(DevParams P, StatePtrs st, 
   for (int t = 0; t < M; ++t) act_cnt[t] = 0;
   double inv_lam_k = 1.0;
 
+  CapSched csch(P, k0call);
 #pragma unroll 1
   for (int kk = 0; kk < Ktot; ++kk) {
     const int64_t k = k0call + kk;
-    const double cap = gen_cap_at(cap_base, k, P.cap_period, P.cap_lo, P.cap_hi, P.cap_mult);
+    const double cap = csch.cap(P, cap_base);
+    csch.next(P);
+    // ---- S4's draws first (burst epoch, demand and meter noise of period
+    // k + 1): they depend only on the seeds, so their integer hash chain
+    // overlaps the FP64 chain of S1-S3 below instead of following it
+    if (left == 0) {
+      ++epoch;
+      left = GEN_BURST_HOLD;
+      bmask = 0u;
+      if (P.demand_kind != 0) {
+        uint64_t sb = gen_period_seed(kburst, epoch);
+#pragma unroll
+        for (int q = 0; q < N; ++q) {
+          sb = gen_lcg(sb);
+          bmask |= ((uint32_t)(sb >> 32) < 858993460u ? 1u : 0u) << q;
+        }
+      }
+    }
+    --left;
+    const uint64_t hper = gen_period_seed(kjit, k + 1);
+    const double dem = P.demand_kind == 0
+                           ? gen_demand_const(tm, P.demand_frac)
+                           : gen_demand_u(gen_jit_v(hper * jump_a + jump_c, j), (bmask >> j) & 1u, tm, bas, amp);
+    const double noise = gen_noise_h(hper, P.noise_scale);
     if ((kk & P.fold_mask) == P.fold_mask) {  // fold lam^-kk back into Sigma' (as slab_rescale)
       const double f = rcp_fast(inv_lam_k);
 #pragma unroll
@@ -309,25 +333,7 @@ __global__ void __launch_bounds__(128) k_simulate_lp(DevParams P, StatePtrs st, 
         }
       }
     }
-    // ---- S4 (own knob): burst epoch, demand, plant
-    if (left == 0) {
-      ++epoch;
-      left = GEN_BURST_HOLD;
-      bmask = 0u;
-      if (P.demand_kind != 0) {
-        uint64_t sb = gen_period_seed(kburst, epoch);
-#pragma unroll
-        for (int q = 0; q < N; ++q) {
-          sb = gen_lcg(sb);
-          bmask |= ((uint32_t)(sb >> 32) < 858993460u ? 1u : 0u) << q;
-        }
-      }
-    }
-    --left;
-    const uint64_t hper = gen_period_seed(kjit, k + 1);
-    const double dem = P.demand_kind == 0
-                           ? gen_demand_const(tm, P.demand_frac)
-                           : gen_demand_u(gen_jit_v(hper * jump_a + jump_c, j), (bmask >> j) & 1u, tm, bas, amp);
+    // ---- S4 (own knob): plant (the draws were formed at the top of the period)
     if (slot >= 0 && ivalid && own && tr.levels) {
       const GridEntry *tab = P.grid + kc.cls * kMaxL;
       double a2 = ac;
@@ -340,7 +346,6 @@ __global__ void __launch_bounds__(128) k_simulate_lp(DevParams P, StatePtrs st, 
     }
     plant_knob<S>(P, kc, u0j, ac, dem, tm, fb, th_r);
     lp_gather<N, G>(fb, fba);
-    const double noise = gen_noise_h(hper, P.noise_scale);
     double pw = c_true;
 #pragma unroll
     for (int q = 0; q < N; ++q) pw = fma(ATa[q], fba[q], pw);

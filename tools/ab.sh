@@ -11,7 +11,7 @@ for rep in $(seq 1 ${REPS:-2}); do
 for v in ${VARIANTS:-base prod}; do
   lv=$v; [ "$v" = "prod" ] && lv=""
   for c in ${CFGS:-3 5}; do
-    extra=""; [ "$c" = "5" ] && extra="--periods 500"; [ "$c" = "4" ] && extra="--periods 200"
+    extra=""; [ "$c" = "5" ] && extra="--periods 500"; [ "$c" = "4" ] && extra="--periods 200"; [ "$c" = "slo" ] && extra="--periods 400"
     CAPGPU_LIB_VARIANT=$lv timeout 300 python bench.py --config $c --no-cpu-baseline --steps ${STEPS:-5} --warmup 3 $extra > gpurun_out/ab${c}_$v.json 2>gpurun_out/ab${c}_$v.err; show gpurun_out/ab${c}_$v.json "cfg$c lib=$v"
   done
 done
