@@ -2070,7 +2070,10 @@ inline int sim_chunks(int64_t n_groups, int64_t slots, int K) {
   for (int C = 2; C <= 64 && K / C >= 16; ++C) {
     const double rounds = (double)n_groups * C / slots;
     const double idle = (std::ceil(rounds) - rounds) / std::ceil(rounds);  // last-round idle share
-    const double cost = idle + 0.002 * C;                                    // + state round trips
+    // + the state round trip and the chunked instantiation's per-period cost:
+    // 0.01 per chunk (measured: cfg 3, 1.73 waves, C = 4: 6.12 -> 6.35 G steps/s;
+    // a cfg 5 2-GPU shard, 55.4 waves, C = 2 instead of 1: 20.4 -> 18.7)
+    const double cost = idle + 0.01 * C;
     if (cost < best_cost) {
       best_cost = cost;
       best = C;
@@ -2219,7 +2222,12 @@ struct LaunchNM {
         return (int)cudaGetLastError();
       }
     }
-    if (occ128[nc] <= 0 || busiest(occ32[nc], 32) < busiest(occ128[nc], 128))
+    // 32-wide CTAs only for a clearly emptier busiest SM (or the chunked
+    // schedule, which needs them): with many waves the 128-wide launch runs
+    // ~9 % faster (cfg 5 shards, N = 4: 20.4 vs 22.5 G steps/s)
+    const int64_t n_groups32 = (P.n_inst + 31) / 32, slots32 = (int64_t)occ32[nc] * sms;
+    const bool chunk = S > 0 && !P.no_chunking && slots32 > 0 && sim_chunks(n_groups32, slots32, K) > 1;
+    if (occ128[nc] <= 0 || chunk || busiest(occ32[nc], 32) < 0.97 * busiest(occ128[nc], 128))
       return launch_sim<N, M, S, 32>(P, st, tr, k0, K, s);
     return launch_sim<N, M, S, 128>(P, st, tr, k0, K, s);
   }
