@@ -659,13 +659,14 @@ struct SimOccupancy {
 #else
   static constexpr int warps = N <= 4 ? 16 : (N <= 6 ? 12 : 8);
 #endif
-  // The SLO-schedule instantiation (general block solve, out-of-line exact
-  // fallback) spills at 128 registers: 12 warps (168 registers) measured
-  // 10.42 vs 8.71 G steps/s at 16 and 9.29 at 8 (N = 4, tools/ab_slo.sh).
+  // The SLO-schedule instantiation (general block solve): with Newton + the
+  // out-of-line fallback it spilled at 128 registers and ran best at 12 warps
+  // (10.42 vs 8.71 G steps/s at 16, N = 4); with the branch-free block_direct
+  // solve 16 warps are best again (12.97 vs 12.84 G at 12, tools/ab.sh).
 #ifdef CAPGPU_SLO_WARPS
   static constexpr int slo_warps = CAPGPU_SLO_WARPS < warps ? CAPGPU_SLO_WARPS : warps;
 #else
-  static constexpr int slo_warps = warps < 12 ? warps : 12;
+  static constexpr int slo_warps = warps;
 #endif
 };
 
