@@ -193,11 +193,11 @@ int budget_reduce(Budget **bs, int n, bool /*consts*/, cudaStream_t s, char *err
   const int64_t cnt = 2 * bs[0]->nb_g;
   if (n == 1) {
     Budget &b = *bs[0];
-    if (b.world > 1) {
-      if (!b.comm) {
-        snprintf(err, 512, "world > 1 needs an NCCL communicator (capgpu_shard.use_nccl) or simulate_group");
-        return CAPGPU_E_INVALID;
-      }
+    if (b.world > 1 && !b.comm) {
+      snprintf(err, 512, "world > 1 needs an NCCL communicator (capgpu_shard.use_nccl) or simulate_group");
+      return CAPGPU_E_INVALID;
+    }
+    if (b.comm) {  // any communicator, also a one-rank one (the single-GPU test of the NCCL path)
       ncclResult_t r = ncclAllReduce(b.send, b.recv, (size_t)cnt, ncclDouble, ncclSum, (ncclComm_t)b.comm, s);
       if (r != ncclSuccess) {
         snprintf(err, 512, "ncclAllReduce: %s", ncclGetErrorString(r));

@@ -1528,7 +1528,10 @@ __device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs 
     double dem[N], thr_max[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) thr_max[j] = TMa.get(j);
-    demand_all<N>(P, gen_stream_key(P.seed, GEN_TAG_JIT, srv), k + 1, bm, thr_max, BAa, AMa, dem);
+    // one period seed for the demand jitter and the meter noise of period k + 1
+    // (gen_noise(key, b) = gen_noise_h(gen_period_seed(key, b)): same draws)
+    const uint64_t hper = gen_period_seed(gen_stream_key(P.seed, GEN_TAG_JIT, srv), k + 1);
+    demand_h<N>(P, hper, bm, thr_max, BAa, AMa, dem);
     if (slot >= 0 && tr.levels) {
       double u_l[N], a_l[N];
 #pragma unroll
@@ -1543,7 +1546,7 @@ __device__ __forceinline__ void period_body(const DevParams &P, const StatePtrs 
       plant_pair<N, SS>(P, u0, acc, dem, thr_max, fbar, thr);
     else
       plant_delta_sigma<N>(P, P.grid, u0, acc, dem, thr_max, fbar, thr);
-    const double noise = gen_noise(gen_stream_key(P.seed, GEN_TAG_JIT, srv), k + 1, P.noise_scale);
+    const double noise = gen_noise_h(hper, P.noise_scale);
     double pw = PT::ro ? tile[PT::oCT * 32] : st.c_true[i];
 #pragma unroll
     for (int j = 0; j < N; ++j) pw = fma(ATa.get(j), fbar[j], pw);

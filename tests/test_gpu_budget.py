@@ -45,6 +45,28 @@ def test_hierarchical_vs_oracle(G, oracle_mod, ref_alpha):
     np.testing.assert_allclose(out["final_p"], ref["final_p"], rtol=0, atol=1e-6)
 
 
+def test_nccl_one_rank_bitwise(G):
+    """The library's NCCL path on one GPU: a one-rank communicator created by
+    capgpu_create from capgpu_nccl_unique_id (ncclCommInitRank) and the
+    per-period ncclAllReduce of the padded block vector (inside the CUDA graph
+    of the period loop) give results bitwise identical to the communicator-free
+    identity reduction."""
+    import os
+    os.environ.setdefault("NCCL_SOCKET_IFNAME", "lo")  # the bootstrap needs no network for one rank
+    d = _desc(40)
+    wl = G.workload_from(d)
+    n = 2048
+    trs = np.array([3, 1500])
+    plain = G.CapGPU.from_config(d, n_servers=n, n_servers_global=n)
+    o1 = {k: H(v) for k, v in plain.simulate(40, wl, trace_inst=trs).items()}
+    nc = G.CapGPU.from_config(d, n_servers=n, n_servers_global=n, world=1, rank=0, nccl_id=G.nccl_unique_id())
+    o2 = {k: H(v) for k, v in nc.simulate(40, wl, trace_inst=trs).items()}
+    for k in ("agg_W", "agg_P", "tr_p", "tr_cap", "final_p", "sum_p"):
+        assert np.array_equal(o1[k], o2[k]), k
+    nc.close()
+    plain.close()
+
+
 @pytest.mark.parametrize("shards", [2, 4, 8])
 def test_shard_invariance_bitwise(G, shards):
     """1 GPU holding all servers == `shards` loopback shards (same device):
