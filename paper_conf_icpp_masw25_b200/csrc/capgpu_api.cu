@@ -701,6 +701,11 @@ static int sim_validate(capgpu_ctx *c, const capgpu_workload *wl, const capgpu_t
     return fail(c, CAPGPU_E_INVALID, "cap schedule");
   if (wl->hierarchical && c->prm.caps_per_server != 1)
     return fail(c, CAPGPU_E_INVALID, "hierarchical budget needs caps_per_server == 1");
+  if (wl->hierarchical && (wl->rack < 1 || wl->rack > 32 || (wl->rack & (wl->rack - 1)) != 0))
+    return fail(c, CAPGPU_E_INVALID, "rack must be a power of two <= 32");
+  if (wl->hierarchical && (c->shard.n_servers_global % wl->rack != 0 || c->n_srv % wl->rack != 0))
+    return fail(c, CAPGPU_E_INVALID, "server count %lld (shard %lld) is not a multiple of the rack size %d (Q16)",
+                (long long)c->shard.n_servers_global, (long long)c->n_srv, wl->rack);
   if (!std::isfinite(wl->gain_dlo) || !std::isfinite(wl->gain_step))
     return fail(c, CAPGPU_E_INVALID, "gain_dlo / gain_step must be finite");
   if (wl->hierarchical && (wl->gain_dlo != 0.0 || wl->gain_step != 0.0))

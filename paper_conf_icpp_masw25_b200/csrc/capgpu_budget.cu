@@ -127,6 +127,11 @@ int budget_alloc(Budget &b, const DevParams &P, const capgpu_workload &wl, const
     snprintf(err, 512, "rack must be a power of two <= 32");
     return CAPGPU_E_INVALID;
   }
+  if (sh.n_servers_global % wl.rack != 0 || P.n_srv % wl.rack != 0) {  // whole racks (Q16; the oracle's rule too)
+    snprintf(err, 512, "server count %lld (shard %lld) is not a multiple of the rack size %d",
+             (long long)sh.n_servers_global, (long long)P.n_srv, wl.rack);
+    return CAPGPU_E_INVALID;
+  }
   if (wl.block != 0 && wl.block != kBudgetBlock) {
     snprintf(err, 512, "reduction block must be %d servers", kBudgetBlock);
     return CAPGPU_E_UNSUPPORTED;

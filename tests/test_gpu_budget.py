@@ -45,6 +45,31 @@ def test_hierarchical_vs_oracle(G, oracle_mod, ref_alpha):
     np.testing.assert_allclose(out["final_p"], ref["final_p"], rtol=0, atol=1e-6)
 
 
+@pytest.mark.parametrize("n", [1040, 1041])
+def test_hierarchical_ragged_and_odd(G, oracle_mod, n):
+    """Server counts off the 32-server warp grid: 1040 (even: the last warp's
+    TMA boxes run past n_srv and are zero-filled, those lanes store nothing)
+    and 1041 with racks of one server (odd: 8-byte rows are not 16-byte
+    aligned, so k_period stages with per-thread cp.async instead of tensor
+    maps) -- both against the oracle.  A server count that is not a whole
+    number of racks is rejected before any launch."""
+    d = _desc(40)
+    if n % 16:
+        with pytest.raises(G.CapGPUError, match="rack"):
+            G.CapGPU.from_config(d, n_servers=n, n_servers_global=n).simulate(1, G.workload_from(d))
+        d["workload"]["rack"] = 1
+    trs = np.array([0, n // 2, n - 1])
+    g = G.CapGPU.from_config(d, n_servers=n, n_servers_global=n)
+    out = {k: H(v) for k, v in g.simulate(40, G.workload_from(d), trace_inst=trs).items()}
+    ref = oracle_mod.Oracle(d).simulate_hier(n, trs, periods=40)
+    np.testing.assert_allclose(out["agg_W"], ref["agg_W"], rtol=1e-12)
+    np.testing.assert_allclose(out["agg_P"], ref["agg_P"], rtol=1e-12)
+    np.testing.assert_allclose(out["tr_cap"], ref["cap"], rtol=1e-10)
+    np.testing.assert_allclose(out["tr_p"], ref["p"], rtol=0, atol=1e-6)
+    assert np.array_equal(out["tr_levels"], np.transpose(ref["levels"], (0, 2, 3, 1)))
+    np.testing.assert_allclose(out["final_p"], ref["final_p"], rtol=0, atol=1e-6)
+
+
 def test_nccl_one_rank_bitwise(G):
     """The library's NCCL path on one GPU: a one-rank communicator created by
     capgpu_create from capgpu_nccl_unique_id (ncclCommInitRank) and the
