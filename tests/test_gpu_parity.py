@@ -163,6 +163,51 @@ def test_control_step_sequence(G, oracle_mod, n_gpus, P, M, n):
     assert n_tie == 0
 
 
+@pytest.mark.parametrize("n_gpus,M", [(2, 2), (4, 2), (5, 3), (8, 3)])
+def test_control_step_general_bounds(G, oracle_mod, n_gpus, M):
+    """SLO-raised lower bounds l_j > m_j = f_min (Eq. 10b-c): the general block
+    solve on random measurements -- block_direct (all 2N breakpoints at once)
+    for N <= 6, Newton + the breakpoint fallback for N = 9 -- every block's u
+    and codes against the oracle's dense stacked QP with the same box."""
+    d = desc_for(n_gpus, P=8, M=M)
+    for j, k in enumerate(d["knobs"]):
+        if j >= 1:
+            k["f_lo"] = 600.0 + 35.0 * j
+    o = oracle_mod.Oracle(d)
+    N = o.n
+    n = 160
+    rng = np.random.default_rng(11 + N)
+    g = G.CapGPU.from_config(d, n_servers=n)
+    A0 = np.abs(np.where(np.arange(N)[:, None] == 0, 0.05, 0.2) * (1 + 0.2 * rng.standard_normal((N, n)))) + 1e-3
+    g.set_prior(T(A0))
+    models = [o.model_new() for _ in range(n)]
+    fmin, hi = (np.array([k[x] for k in d["knobs"]]) for x in ("f_min", "f_max"))
+    lo = np.array([k.get("f_lo", k["f_min"]) for k in d["knobs"]])
+    tm = 40 + 160 * rng.random((N, n))
+    n_tie = 0
+    for step in range(10):
+        f = fmin[:, None] + (hi - fmin)[:, None] * rng.random((N, n))
+        a_true = np.where(np.arange(N)[:, None] == 0, 0.05, 0.2)
+        p = 300 + np.sum(a_true * f, axis=0) + rng.normal(0, 11, n)
+        thr = tm * rng.random((N, n)) * 1.1
+        pmin = 300 + a_true[:, 0] @ lo; pmax = 300 + a_true[:, 0] @ hi
+        cap = pmin + rng.uniform(-0.1, 1.1, n) * (pmax - pmin)
+        out = g.control_step(T(p), T(f), T(thr), T(tm), T(cap))
+        u, act, ah = (H(out[k]) for k in ("u", "active", "ahat"))
+        for s in range(n):
+            o.model_push(models[s], f[:, s], p[s])
+            aho = o.model_solve(models[s], A0[:, s])
+            np.testing.assert_allclose(ah[:, s], aho, rtol=RTOL, atol=1e-15)
+            _, Ro, _ = o.weights(thr[:, s], tm[:, s])
+            beta = p[s] - cap[s] - aho @ f[:, s]
+            uo, acto, tie, _, _ = o.mpc(aho, Ro, beta, lo, hi, fmin)
+            np.testing.assert_allclose(u[:, :, s], uo, rtol=RTOL, atol=1e-9)
+            bad, ties = active_equal(act[:, s], acto, tie)
+            assert bad == 0, (step, s, act[:, s], acto)
+            n_tie += ties
+    assert n_tie == 0
+
+
 def test_control_step_nonfinite_and_order(G):
     d = desc_for(2)
     g = G.CapGPU.from_config(d, n_servers=8)
