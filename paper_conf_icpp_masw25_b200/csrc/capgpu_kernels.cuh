@@ -2068,16 +2068,21 @@ struct LaunchN {
 // per-chunk state round trip (~2 KB per instance) stays small against a chunk.
 inline int sim_chunks(int64_t n_groups, int64_t slots, int K) {
   if (n_groups <= slots || K < 64) return 1;
-  int best = 1;
   const double r1 = (double)n_groups / slots;
-  double best_cost = (std::ceil(r1) - r1) / std::ceil(r1);  // C = 1: the plain launch
+  // many waves: the plain launch is balanced enough, and the chunked schedule
+  // needs 32-wide CTAs (cfg 5 shards, 55 waves: 128-wide plain 22.5 vs 32-wide
+  // chunked 18.7 G steps/s)
+  if ((std::ceil(r1) - r1) / std::ceil(r1) < 0.05) return 1;
+  // cost of C chunks: last-round idle + the tail (about half a chunk of every
+  // slot idles at the end) + the per-chunk state round trip.  cfg 3 (1.73
+  // waves) measured C = 2 / 4 / 8 / 12 / 16: 5.83 / 6.33 / 6.53 / 6.57 / 6.56 G
+  // steps/s (tools/exp_chunks.sh); this picks 16.
+  int best = 1;
+  double best_cost = 1e30;
   for (int C = 2; C <= 64 && K / C >= 16; ++C) {
-    const double rounds = (double)n_groups * C / slots;
-    const double idle = (std::ceil(rounds) - rounds) / std::ceil(rounds);  // last-round idle share
-    // + the state round trip and the chunked instantiation's per-period cost:
-    // 0.01 per chunk (measured: cfg 3, 1.73 waves, C = 4: 6.12 -> 6.35 G steps/s;
-    // a cfg 5 2-GPU shard, 55.4 waves, C = 2 instead of 1: 20.4 -> 18.7)
-    const double cost = idle + 0.01 * C;
+    const double rounds = r1 * C;
+    const double idle = (std::ceil(rounds) - rounds) / std::ceil(rounds);
+    const double cost = idle + 0.5 / rounds + 0.001 * C;
     if (cost < best_cost) {
       best_cost = cost;
       best = C;
@@ -2128,6 +2133,10 @@ int launch_sim(const DevParams &P, const StatePtrs &st, const TracePtrs &tr, int
       slots = (int64_t)occ * sms;
     }
     C = (st.sched && slots > 0 && !P.no_chunking) ? sim_chunks(n_groups, slots, K) : 1;
+    if (C > 1) {  // experiment override of the chunk count (CAPGPU_SIM_CHUNKS=c)
+      static const char *ce = getenv("CAPGPU_SIM_CHUNKS");
+      if (ce && atoi(ce) > 1) C = std::min(atoi(ce), K / 16);
+    }
     if (C > 1) {
       SimSched sc{};
       sc.ctr = st.sched;
